@@ -1,0 +1,186 @@
+/*
+ * lmo.h -- C ABI of the B200-native (sm_100a) LM-Offload hot path.
+ *
+ * Paper: "LM-Offload: Performance Model-Guided Generative Inference of Large
+ * Language Models with Parallelism Control" (dblp/paper_conf_ipps_wurypgll25).
+ * "P:n" cites line n of the paper text.
+ *
+ * Conventions (all entry points):
+ *  - Every pointer except `cache` / status-string results is a DEVICE
+ *    pointer owned by the caller.  The library never allocates, frees or
+ *    synchronizes; it keeps no mutable global state except a launch counter
+ *    and a once-initialised device-property cache.
+ *  - `stream` is a cudaStream_t passed as void* (0 = legacy default stream).
+ *    Every call only enqueues work on it and returns.
+ *  - Argument errors are detected synchronously BEFORE any launch and nothing
+ *    is written.  A failed launch returns LMO_ERR_CUDA (cudaGetLastError);
+ *    asynchronous faults surface at the caller's next synchronization.
+ *  - fp16 data is IEEE binary16.  Inputs must be finite (NaN/Inf: results
+ *    unspecified).  No aliasing between inputs and outputs except the KV
+ *    cache, which append updates in place.
+ *  - Storage format ("compressed tensor", Alg 2): 4-bit codes, two
+ *    per byte, LOW nibble = element 2j, HIGH nibble = element 2j+1; one
+ *    lmo_qmeta {fp16 min, fp16 scale} per group of 64 consecutive elements
+ *    along the quantize dimension.  Dequantized value = min + code*scale.
+ */
+#ifndef LMO_H_
+#define LMO_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    LMO_OK = 0,
+    LMO_ERR_NULL = 1,         /* a required pointer is NULL                  */
+    LMO_ERR_SHAPE = 2,        /* a size is negative/zero/inconsistent        */
+    LMO_ERR_UNSUPPORTED = 3,  /* bits != 4, group != 64, head_dim not 64/128, */
+                              /* group ratio > 8, ...                          */
+    LMO_ERR_ALIGN = 4,        /* a pointer is not 16-byte aligned            */
+    LMO_ERR_WORKSPACE = 5,    /* workspace missing or too small              */
+    LMO_ERR_CUDA = 6          /* a CUDA runtime call or launch failed        */
+} lmo_status;
+
+typedef enum { LMO_F16 = 0, LMO_F32 = 1 } lmo_dtype;
+
+/* Per-group metadata, 4 bytes: fp16 bit patterns of the group minimum and of
+ * the quantization step scale = RU16(RN32(max - min) / 15).  scale == 0 iff
+ * the group is constant (Eq 10's 0/0 case, reading 1). */
+typedef struct {
+    uint16_t min_f16;
+    uint16_t scale_f16;
+} lmo_qmeta;
+
+/* ---------------------------------------------------------------------------
+ * A1. Group-wise 4-bit quantization -- Alg 2 "Compress(tensor, target_bits,
+ * quantize_dim)" with Eq 10:
+ *     x_quant = round((x - min) / (max - min) * (2^b - 1)),
+ * evaluated as code = min(15, rint(RN32(RN32(x - min) * RN32(1/scale)))).
+ *
+ * x_f16 : fp16 tensor viewed as (outer, n, inner), contiguous.  Groups are
+ *         group_size consecutive elements along n (the quantize_dim); n is
+ *         padded with +0 to n_pad = ceil(n/64)*64 and the pads take part in
+ *         min/max (Alg 2 l.5-6 precede l.9-10).
+ * codes : (outer, n_pad/2, inner) bytes; byte[o][j][i] packs elements 2j
+ *         (low nibble) and 2j+1 (high nibble) of row (o, :, i).
+ * meta  : (outer, n_pad/64, inner) lmo_qmeta.
+ * bits must be 4 and group_size 64 (else LMO_ERR_UNSUPPORTED).  x, codes and
+ * meta must be 16-byte aligned.  outer/n/inner == 0 is a no-op.
+ * ------------------------------------------------------------------------- */
+lmo_status lmo_quantize_groupwise(const void *x_f16, int64_t outer, int64_t n, int64_t inner,
+                                  int bits, int group_size, uint8_t *codes, lmo_qmeta *meta,
+                                  void *stream);
+
+/* ---------------------------------------------------------------------------
+ * A5. Group-wise dequantization -- Eq 11 in step form:
+ *     y = RN16(RN32(code * scale + min)),
+ * bit-exact with the oracle.  Same (outer, n, inner) view as above; y_f16 is
+ * (outer, n, inner) fp16 (padding dropped).  Weights are quantized once and
+ * only dequantized afterwards (Eq 4).
+ * ------------------------------------------------------------------------- */
+lmo_status lmo_dequantize_groupwise(const uint8_t *codes, const lmo_qmeta *meta, int64_t outer,
+                                    int64_t n, int64_t inner, int bits, int group_size,
+                                    void *y_f16, void *stream);
+
+/* One layer's q4 KV cache (caller-owned device memory), layout
+ *   k_codes, v_codes : [batch][kv_heads][capacity][head_dim/2]  bytes
+ *   k_meta,  v_meta  : [batch][kv_heads][capacity][head_dim/64] lmo_qmeta
+ * i.e. token-major per (sequence, kv head), so a run of tokens is one
+ * contiguous span (one bulk copy).  Groups lie along head_dim (DESIGN.md
+ * reading 8), so every token's groups are self-contained.
+ * head_dim must be 64 or 128; capacity must be a multiple of 16 (callers
+ * round up; the 16-token block is the kernels' unit of work). */
+typedef struct {
+    uint8_t *k_codes;
+    uint8_t *v_codes;
+    lmo_qmeta *k_meta;
+    lmo_qmeta *v_meta;
+    int32_t batch;
+    int32_t kv_heads;
+    int32_t capacity;
+    int32_t head_dim;
+} lmo_kv_cache;
+
+/* ---------------------------------------------------------------------------
+ * A2. KV append-quantize -- "The KV cache is updated by concatenating the
+ * current token's key and value vectors with the existing ones"; "the
+ * newly generated KV cache is quantized" each token, each layer (P:235,
+ * Eq 7; "new KV cache is compressed, old ... only decompressed").
+ *
+ * k_new_f16, v_new_f16 : [batch][kv_heads][n_new][head_dim] fp16.
+ * Row (b, h, t) is quantized exactly as lmo_quantize_groupwise(outer=1,
+ * n=head_dim, inner=1) would, and written to cache slot pos_b + t, where
+ * pos_b = pos_dev[b] if pos_dev != NULL (device int32[batch]) else pos0.
+ * Only slots [pos_b, pos_b + n_new) of each (b, h) are written.
+ * Host-checked: 0 <= pos0, pos0 + n_new <= capacity (when pos_dev == NULL).
+ * With pos_dev, out-of-range rows (pos_b < 0 or pos_b + n_new > capacity)
+ * are skipped on the device.
+ * ------------------------------------------------------------------------- */
+lmo_status lmo_kv_append_quant(const lmo_kv_cache *cache, const void *k_new_f16,
+                               const void *v_new_f16, int32_t n_new, int32_t pos0,
+                               const int32_t *pos_dev, void *stream);
+
+/* Workspace bytes lmo_decode_attention_q4 needs for this shape.  The first
+ * 4*batch*kv_heads bytes are per-(sequence, kv head) arrival counters that
+ * MUST be zero before the first call on a workspace (e.g. cudaMemsetAsync);
+ * every call leaves them zero again.  One call in flight per workspace. */
+size_t lmo_decode_attention_workspace_bytes(int32_t batch, int32_t kv_heads, int32_t q_heads,
+                                            int32_t head_dim, int32_t num_splits);
+
+/* ---------------------------------------------------------------------------
+ * A3+A4. Decode-step attention over the q4 cache with dequantization fused
+ * ("QK^T/sqrt(d_k) ... A softmax function is then applied"; the old
+ * cache is only dequantized, Eq 6):
+ *   o[b][h] = softmax(softmax_scale * q[b][h] . K[b][kvh][0:L_b]^T) V[b][kvh][0:L_b]
+ * with kvh = h / (q_heads / kv_heads) and K/V the dequantized cache rows
+ * (min + code*scale).  fp32 accumulation, numerically stable softmax.
+ *
+ * q_f16       : [batch][q_heads][head_dim] fp16.
+ * len         : L_b for every sequence when seq_lens_dev == NULL
+ *               (1 <= len <= capacity, host-checked).
+ * seq_lens_dev: optional device int32[batch]; L_b = min(seq_lens_dev[b],
+ *               capacity); L_b <= 0 writes a zero output row.
+ * num_splits  : 0 = auto (stream-K: the sequence blocks of all (b, kvh) pairs
+ *               are divided evenly over the resident warps, partial results
+ *               merged in-kernel by the last arriving warp);  k > 0 = each
+ *               (b, kvh) pair is split into k contiguous parts (results then
+ *               independent of batch composition).
+ * out         : [batch][q_heads][head_dim], LMO_F32 or LMO_F16.
+ * q_heads/kv_heads must be in 1..8.
+ * ------------------------------------------------------------------------- */
+lmo_status lmo_decode_attention_q4(const lmo_kv_cache *cache, const void *q_f16, int32_t q_heads,
+                                   int32_t len, const int32_t *seq_lens_dev, float softmax_scale,
+                                   int32_t num_splits, void *out, lmo_dtype out_dtype,
+                                   void *workspace, size_t workspace_bytes, void *stream);
+
+/* Human-readable name of a status code (static string). */
+const char *lmo_status_string(lmo_status status);
+
+/* ---------------------------------------------------------------------------
+ * Support entry points (not steps of the method).
+ * ------------------------------------------------------------------------- */
+
+/* Seeded synthetic inputs (bench/test support, no method arithmetic): fills
+ * dst [nb][nh][npos][dim] fp16 with the counter-based generator documented in
+ * paper_conf_ipps_wurypgll25_b200/inputs.py, at global coordinates
+ * (layer, b0+ib, h0+ih, p0+ip, i).  `group` maps a head to its kv head for
+ * the outlier-channel mask (q: q_heads/kv_heads, K/V: 1).  Bit-identical to
+ * inputs.gen_f16. */
+lmo_status lmo_gen_fill_f16(void *dst, int32_t nb, int32_t nh, int32_t npos, int32_t dim,
+                            uint64_t seed, int32_t stream_id, int32_t layer, int32_t b0,
+                            int32_t h0, int32_t p0, int32_t group, void *stream);
+
+/* Number of kernels this library has launched in this process. */
+uint64_t lmo_launch_count(void);
+
+/* ABI version: (major << 16) | minor. */
+uint32_t lmo_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* LMO_H_ */

@@ -1,0 +1,169 @@
+// common.cuh -- sm_100a device helpers shared by the liblmo kernels.
+// (Product code.  Shares nothing with oracle/.)
+#pragma once
+
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "lmo.h"
+
+namespace lmo {
+
+constexpr int kGroup = 64;   // quantization group (elements)
+constexpr int kQMax = 15;    // 2^b - 1, b = 4
+
+// ------------------------------------------------------------ launch stats
+void note_launch();                         // lmo_abi.cu
+int device_sm_count();                      // cached per device
+
+// ------------------------------------------------------- quantization math
+// One rounding chain, identical in every kernel that quantizes (K1, K2):
+//   range = RN32(mx - mn); scale = RU16(RU32(range / 15)) == RU16(range/15);
+//   inv = scale == 0 ? 0 : RN32(1/scale);
+//   code = min(15, rint_even(RN32(RN32(x - mn) * inv))).
+struct GroupParams {
+    float mn;       // canonical (+0 for a zero min)
+    float inv;
+    __half mn_h;
+    __half scale_h;
+};
+
+__device__ __forceinline__ GroupParams group_params(float mn, float mx) {
+    GroupParams p;
+    p.mn = __fadd_rn(mn, 0.0f);                         // -0 -> +0
+    float range = __fsub_rn(__fadd_rn(mx, 0.0f), p.mn);
+    p.scale_h = __float2half_ru(__fdiv_ru(range, 15.0f));
+    float s = __half2float(p.scale_h);
+    p.inv = (s == 0.0f) ? 0.0f : __frcp_rn(s);
+    p.mn_h = __float2half_rn(p.mn);                     // exact: mn is an fp16 value
+    return p;
+}
+
+__device__ __forceinline__ uint32_t quant_code(float x, const GroupParams &p) {
+    float d = __fsub_rn(x, p.mn);
+    float t = __fmul_rn(d, p.inv);
+    // rint half-even for 0 <= t < 2^22: add 1.5*2^23, read the low mantissa bits
+    float r = __fadd_rn(t, 12582912.0f);
+    uint32_t c = __float_as_uint(r) - 0x4B400000u;
+    return c > 15u ? 15u : c;
+}
+
+__device__ __forceinline__ uint32_t meta_word(const GroupParams &p) {
+    return (uint32_t)__half_as_ushort(p.mn_h) | ((uint32_t)__half_as_ushort(p.scale_h) << 16);
+}
+
+// Quantize one 64-group held by 8 consecutive lanes (lane8 = lane & 7), each
+// holding 8 consecutive fp16 elements (16 B).  Returns this lane's 4 code
+// bytes (elements 8*lane8 .. 8*lane8+7) and, via `meta`, the group meta word.
+__device__ __forceinline__ uint32_t quantize_group_lane8(const uint4 xv, uint32_t &meta) {
+    const __half2 *h2 = reinterpret_cast<const __half2 *>(&xv);
+    float v[8];
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        float2 f = __half22float2(h2[k]);
+        v[2 * k] = f.x;
+        v[2 * k + 1] = f.y;
+    }
+    float mn = v[0], mx = v[0];
+#pragma unroll
+    for (int k = 1; k < 8; ++k) {
+        mn = fminf(mn, v[k]);
+        mx = fmaxf(mx, v[k]);
+    }
+#pragma unroll
+    for (int off = 1; off < 8; off <<= 1) {
+        mn = fminf(mn, __shfl_xor_sync(0xffffffffu, mn, off));
+        mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+    }
+    GroupParams p = group_params(mn, mx);
+    uint32_t w = 0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) w |= quant_code(v[k], p) << (4 * k);
+    meta = meta_word(p);
+    return w;
+}
+
+// ------------------------------------------------------------- PTX wrappers
+__device__ __forceinline__ uint32_t smem_u32(const void *p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(count));
+}
+
+__device__ __forceinline__ void fence_mbar_init() {
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(smem_u32(bar)),
+                 "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity) {
+    uint32_t addr = smem_u32(bar);
+    asm volatile(
+        "{\n"
+        ".reg .pred P1;\n"
+        "LAB_WAIT:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+        "@P1 bra DONE;\n"
+        "bra LAB_WAIT;\n"
+        "DONE:\n"
+        "}\n" ::"r"(addr),
+        "r"(parity)
+        : "memory");
+}
+
+// 1-D bulk async copy global -> shared (TMA engine, SASS UBLKCP), completion
+// counted on an mbarrier.  size and both addresses must be 16-B aligned.
+__device__ __forceinline__ void bulk_g2s(void *smem_dst, const void *gmem_src, uint32_t bytes,
+                                         uint64_t *bar, uint64_t policy) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint "
+        "[%0], [%1], %2, [%3], %4;\n" ::"r"(smem_u32(smem_dst)),
+        "l"(gmem_src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy)
+        : "memory");
+}
+
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;\n" : "=l"(pol));
+    return pol;
+}
+
+// D(16x8, f32) += A(16x16, f16, row) * B(16x8, f16, col)   [HMMA]
+__device__ __forceinline__ void mma_16816(float (&c)[4], uint32_t a0, uint32_t a1, uint32_t a2,
+                                          uint32_t a3, uint32_t b0, uint32_t b1) {
+    asm("mma.sync.aligned.m16n8k16.row.col.f32.f16.f16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, "
+        "{%8,%9}, {%0,%1,%2,%3};\n"
+        : "+f"(c[0]), "+f"(c[1]), "+f"(c[2]), "+f"(c[3])
+        : "r"(a0), "r"(a1), "r"(a2), "r"(a3), "r"(b0), "r"(b1));
+}
+
+__device__ __forceinline__ uint32_t lop3_and_or(uint32_t x, uint32_t mask, uint32_t orv) {
+    uint32_t r;
+    asm("lop3.b32 %0, %1, %2, %3, 0xEA;\n" : "=r"(r) : "r"(x), "r"(mask), "r"(orv));  // (x&m)|o
+    return r;
+}
+
+__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
+    uint32_t r;
+    asm("prmt.b32 %0, %1, %2, %3;\n" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
+    return r;
+}
+
+__device__ __forceinline__ uint32_t hsub2_u32(uint32_t a, uint32_t b) {
+    __half2 r = __hsub2(*reinterpret_cast<__half2 *>(&a), *reinterpret_cast<__half2 *>(&b));
+    return *reinterpret_cast<uint32_t *>(&r);
+}
+
+__device__ __forceinline__ uint32_t pack_half2(float lo, float hi) {
+    __half2 h = __floats2half2_rn(lo, hi);
+    return *reinterpret_cast<uint32_t *>(&h);
+}
+
+}  // namespace lmo

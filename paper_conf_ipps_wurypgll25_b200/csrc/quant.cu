@@ -1,0 +1,210 @@
+// quant.cu -- K1 group-wise quantize (Alg 2 / Eq 10), K2 KV append-quantize
+// (Eq 7), K5 group-wise dequantize (Eq 11).  sm_100a.
+//
+// All three are HBM-streaming kernels (2.5625 B/element moved for K1/K2,
+// 2.5625 for K5): 128-bit coalesced loads/stores, 8 lanes per 64-group,
+// warp-shuffle min/max, no shared memory.  The rounding chain lives in
+// common.cuh (group_params / quant_code) and is the same for K1 and K2, so
+// append is bit-identical to quantize on the same rows by construction.
+#include "common.cuh"
+
+namespace lmo {
+
+__device__ __forceinline__ uint4 ldg_stream(const void *p) {
+    uint4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];\n"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+                 : "l"(p));
+    return r;
+}
+
+// K1 fast path: inner == 1, n % 64 == 0.  One 64-group per 8 lanes.
+__global__ void __launch_bounds__(256) quantize_vec_kernel(const __half *__restrict__ x,
+                                                           int64_t ngroups_total,
+                                                           uint8_t *__restrict__ codes,
+                                                           uint32_t *__restrict__ meta) {
+    const int lane8 = threadIdx.x & 7;
+    const int64_t gid = (int64_t)blockIdx.x * (blockDim.x / 8) + (threadIdx.x >> 3);
+    const bool valid = gid < ngroups_total;
+    uint4 xv = make_uint4(0, 0, 0, 0);
+    if (valid) xv = ldg_stream(x + gid * kGroup + lane8 * 8);
+    uint32_t mw;
+    uint32_t w = quantize_group_lane8(xv, mw);     // all lanes take part in shuffles
+    if (valid) {
+        reinterpret_cast<uint32_t *>(codes + gid * (kGroup / 2))[lane8] = w;
+        if (lane8 == 0) meta[gid] = mw;
+    }
+}
+
+// K1 general path: any (outer, n, inner); one thread per (o, group, i), i
+// fastest so that inner > 1 (e.g. grouping a weight matrix along its output
+// dim) is coalesced across threads.
+__global__ void __launch_bounds__(256) quantize_generic_kernel(const __half *__restrict__ x,
+                                                               int64_t outer, int64_t n,
+                                                               int64_t inner,
+                                                               uint8_t *__restrict__ codes,
+                                                               uint32_t *__restrict__ meta) {
+    const int64_t ng = (n + kGroup - 1) / kGroup;
+    const int64_t total = outer * ng * inner;
+    for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = idx % inner;
+        const int64_t g = (idx / inner) % ng;
+        const int64_t o = idx / (inner * ng);
+        float mn = INFINITY, mx = -INFINITY;
+        for (int k = 0; k < kGroup; ++k) {
+            const int64_t j = g * kGroup + k;
+            const float v = (j < n) ? __half2float(x[(o * n + j) * inner + i]) : 0.0f;
+            mn = fminf(mn, v);
+            mx = fmaxf(mx, v);
+        }
+        const GroupParams p = group_params(mn, mx);
+        const int64_t npad2 = ng * kGroup / 2;
+        for (int k = 0; k < kGroup; k += 2) {
+            const int64_t j = g * kGroup + k;
+            const float v0 = (j < n) ? __half2float(x[(o * n + j) * inner + i]) : 0.0f;
+            const float v1 = (j + 1 < n) ? __half2float(x[(o * n + j + 1) * inner + i]) : 0.0f;
+            codes[(o * npad2 + j / 2) * inner + i] =
+                (uint8_t)(quant_code(v0, p) | (quant_code(v1, p) << 4));
+        }
+        meta[(o * ng + g) * inner + i] = meta_word(p);
+    }
+}
+
+// K2: quantize new K/V rows [B][Hkv][n_new][d] into cache slots pos_b + t.
+// Group id space: kv (2) x B x Hkv x n_new x (d/64), K rows first.
+__global__ void __launch_bounds__(256) kv_append_kernel(lmo_kv_cache cache,
+                                                        const __half *__restrict__ k_new,
+                                                        const __half *__restrict__ v_new,
+                                                        int n_new, int pos0,
+                                                        const int32_t *__restrict__ pos_dev) {
+    const int d = cache.head_dim;
+    const int gpr = d / kGroup;
+    const int lane8 = threadIdx.x & 7;
+    const int64_t rows_per_kv = (int64_t)cache.batch * cache.kv_heads * n_new;
+    const int64_t ngroups = 2 * rows_per_kv * gpr;
+    const int64_t gid = (int64_t)blockIdx.x * (blockDim.x / 8) + (threadIdx.x >> 3);
+    bool valid = gid < ngroups;
+    const int64_t gg = valid ? gid : 0;
+    const int kv = (int)(gg / (rows_per_kv * gpr));
+    const int64_t r = (gg / gpr) % rows_per_kv;          // (b*Hkv + h)*n_new + t
+    const int grp = (int)(gg % gpr);
+    const int t = (int)(r % n_new);
+    const int64_t bh = r / n_new;
+    const int b = (int)(bh / cache.kv_heads);
+    const int pos = pos_dev ? pos_dev[b] : pos0;
+    if (pos < 0 || pos + n_new > cache.capacity) valid = false;
+    const __half *src = (kv == 0 ? k_new : v_new) + r * d + grp * kGroup + lane8 * 8;
+    uint4 xv = make_uint4(0, 0, 0, 0);
+    if (valid) xv = ldg_stream(src);
+    uint32_t mw;
+    const uint32_t w = quantize_group_lane8(xv, mw);
+    if (valid) {
+        const int64_t slot = bh * cache.capacity + pos + t;
+        uint8_t *cdst = (kv == 0 ? cache.k_codes : cache.v_codes) + slot * (d / 2) + grp * 32;
+        uint32_t *mdst = reinterpret_cast<uint32_t *>(kv == 0 ? cache.k_meta : cache.v_meta) +
+                         slot * gpr + grp;
+        reinterpret_cast<uint32_t *>(cdst)[lane8] = w;
+        if (lane8 == 0) *mdst = mw;
+    }
+}
+
+__device__ __forceinline__ __half dequant_one(uint32_t c, uint32_t mw) {
+    const float mn = __half2float(__ushort_as_half((unsigned short)(mw & 0xffffu)));
+    const float sc = __half2float(__ushort_as_half((unsigned short)(mw >> 16)));
+    return __float2half_rn(__fmaf_rn((float)c, sc, mn));   // RN16(RN32(c*scale + min))
+}
+
+// K5 fast path: inner == 1, n % 64 == 0; 8 elements (4 code bytes, 16 B out) per thread.
+__global__ void __launch_bounds__(256) dequantize_vec_kernel(const uint8_t *__restrict__ codes,
+                                                             const uint32_t *__restrict__ meta,
+                                                             int64_t n_oct,
+                                                             __half *__restrict__ y) {
+    const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (idx >= n_oct) return;
+    const uint32_t w = __ldg(reinterpret_cast<const uint32_t *>(codes) + idx);
+    const uint32_t mw = __ldg(meta + idx / 8);
+    uint4 out;
+    uint32_t *o = reinterpret_cast<uint32_t *>(&out);
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const __half lo = dequant_one((w >> (8 * k)) & 0xf, mw);
+        const __half hi = dequant_one((w >> (8 * k + 4)) & 0xf, mw);
+        o[k] = (uint32_t)__half_as_ushort(lo) | ((uint32_t)__half_as_ushort(hi) << 16);
+    }
+    reinterpret_cast<uint4 *>(y)[idx] = out;
+}
+
+// K5 general path: one thread per output element.
+__global__ void __launch_bounds__(256) dequantize_generic_kernel(const uint8_t *__restrict__ codes,
+                                                                 const uint32_t *__restrict__ meta,
+                                                                 int64_t outer, int64_t n,
+                                                                 int64_t inner,
+                                                                 __half *__restrict__ y) {
+    const int64_t ng = (n + kGroup - 1) / kGroup;
+    const int64_t npad2 = ng * kGroup / 2;
+    const int64_t total = outer * n * inner;
+    for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = idx % inner;
+        const int64_t j = (idx / inner) % n;
+        const int64_t o = idx / (inner * n);
+        const uint8_t byte = codes[(o * npad2 + j / 2) * inner + i];
+        const uint32_t c = (j & 1) ? (byte >> 4) : (byte & 0xf);
+        y[idx] = dequant_one(c, meta[(o * ng + j / kGroup) * inner + i]);
+    }
+}
+
+// ------------------------------------------------------------ host launch
+static int grid_for(int64_t work, int per_block) {
+    int64_t g = (work + per_block - 1) / per_block;
+    const int64_t cap = (int64_t)device_sm_count() * 32;
+    return (int)(g < 1 ? 1 : (g > cap ? cap : g));
+}
+
+cudaError_t launch_quantize(const void *x, int64_t outer, int64_t n, int64_t inner,
+                            uint8_t *codes, lmo_qmeta *meta, cudaStream_t st) {
+    const __half *xh = static_cast<const __half *>(x);
+    uint32_t *mw = reinterpret_cast<uint32_t *>(meta);
+    if (inner == 1 && n % kGroup == 0) {
+        const int64_t groups = outer * (n / kGroup);
+        const int64_t blocks = (groups + 31) / 32;
+        quantize_vec_kernel<<<(unsigned)blocks, 256, 0, st>>>(xh, groups, codes, mw);
+    } else {
+        const int64_t work = outer * ((n + kGroup - 1) / kGroup) * inner;
+        quantize_generic_kernel<<<grid_for(work, 256), 256, 0, st>>>(xh, outer, n, inner, codes,
+                                                                       mw);
+    }
+    note_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_dequantize(const uint8_t *codes, const lmo_qmeta *meta, int64_t outer,
+                              int64_t n, int64_t inner, void *y, cudaStream_t st) {
+    const uint32_t *mw = reinterpret_cast<const uint32_t *>(meta);
+    __half *yh = static_cast<__half *>(y);
+    if (inner == 1 && n % kGroup == 0) {
+        const int64_t n_oct = outer * n / 8;
+        dequantize_vec_kernel<<<(unsigned)((n_oct + 255) / 256), 256, 0, st>>>(codes, mw, n_oct,
+                                                                                yh);
+    } else {
+        dequantize_generic_kernel<<<grid_for(outer * n * inner, 256), 256, 0, st>>>(
+            codes, mw, outer, n, inner, yh);
+    }
+    note_launch();
+    return cudaGetLastError();
+}
+
+cudaError_t launch_kv_append(const lmo_kv_cache &cache, const void *k_new, const void *v_new,
+                             int n_new, int pos0, const int32_t *pos_dev, cudaStream_t st) {
+    const int64_t groups =
+        2LL * cache.batch * cache.kv_heads * n_new * (cache.head_dim / kGroup);
+    const int64_t blocks = (groups + 31) / 32;
+    kv_append_kernel<<<(unsigned)blocks, 256, 0, st>>>(cache, static_cast<const __half *>(k_new),
+                                                       static_cast<const __half *>(v_new), n_new,
+                                                       pos0, pos_dev);
+    note_launch();
+    return cudaGetLastError();
+}
+
+}  // namespace lmo

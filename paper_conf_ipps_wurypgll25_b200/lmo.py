@@ -1,0 +1,221 @@
+"""Thin ctypes binding of liblmo.so (include/lmo.h) -- argument marshalling only.
+
+Every step of the path runs in the library's CUDA kernels; this module only
+turns torch tensors into (device pointer, size) arguments, passes the current
+CUDA stream, and raises on a non-OK status.  There is no CPU fallback: if the
+library is missing or cannot be loaded, importing this module raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import math
+import os
+from dataclasses import dataclass
+
+import torch
+
+from . import build as _build
+
+LMO_OK, LMO_ERR_NULL, LMO_ERR_SHAPE, LMO_ERR_UNSUPPORTED, LMO_ERR_ALIGN, LMO_ERR_WORKSPACE, \
+    LMO_ERR_CUDA = range(7)
+LMO_F16, LMO_F32 = 0, 1
+GROUP = 64
+
+
+class LmoError(RuntimeError):
+    def __init__(self, status: int, fn: str):
+        super().__init__(f"{fn}: {_lib.lmo_status_string(status).decode()}")
+        self.status = status
+
+
+class lmo_kv_cache(ctypes.Structure):
+    _fields_ = [("k_codes", ctypes.c_void_p), ("v_codes", ctypes.c_void_p),
+                ("k_meta", ctypes.c_void_p), ("v_meta", ctypes.c_void_p),
+                ("batch", ctypes.c_int32), ("kv_heads", ctypes.c_int32),
+                ("capacity", ctypes.c_int32), ("head_dim", ctypes.c_int32)]
+
+
+def _load():
+    path = _build.LIB
+    if not os.path.exists(path):
+        raise ImportError(f"liblmo.so not built ({path}); run __graft_entry__.build()")
+    L = ctypes.CDLL(path)
+    P, i64, i32, u64 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64
+    sig = {
+        "lmo_quantize_groupwise": [P, i64, i64, i64, ctypes.c_int, ctypes.c_int, P, P, P],
+        "lmo_dequantize_groupwise": [P, P, i64, i64, i64, ctypes.c_int, ctypes.c_int, P, P],
+        "lmo_kv_append_quant": [ctypes.POINTER(lmo_kv_cache), P, P, i32, i32, P, P],
+        "lmo_decode_attention_q4": [ctypes.POINTER(lmo_kv_cache), P, i32, i32, P, ctypes.c_float,
+                                    i32, P, ctypes.c_int, P, ctypes.c_size_t, P],
+        "lmo_gen_fill_f16": [P, i32, i32, i32, i32, u64, i32, i32, i32, i32, i32, i32, P],
+    }
+    for name, args in sig.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = ctypes.c_int
+    L.lmo_decode_attention_workspace_bytes.argtypes = [i32, i32, i32, i32, i32]
+    L.lmo_decode_attention_workspace_bytes.restype = ctypes.c_size_t
+    L.lmo_status_string.argtypes = [ctypes.c_int]
+    L.lmo_status_string.restype = ctypes.c_char_p
+    L.lmo_launch_count.argtypes = []
+    L.lmo_launch_count.restype = ctypes.c_uint64
+    L.lmo_version.argtypes = []
+    L.lmo_version.restype = ctypes.c_uint32
+    return L
+
+
+_lib = _load()
+LIB_PATH = _build.LIB
+EXPORTS = ["lmo_quantize_groupwise", "lmo_dequantize_groupwise", "lmo_kv_append_quant",
+           "lmo_decode_attention_workspace_bytes", "lmo_decode_attention_q4", "lmo_status_string",
+           "lmo_gen_fill_f16", "lmo_launch_count", "lmo_version"]
+
+
+def _check(status: int, fn: str) -> None:
+    if status != LMO_OK:
+        raise LmoError(status, fn)
+
+
+def _ptr(t: torch.Tensor | None):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _stream(stream=None):
+    s = torch.cuda.current_stream() if stream is None else stream
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _need_cuda(*ts):
+    for t in ts:
+        if t is not None and (not t.is_cuda or not t.is_contiguous()):
+            raise ValueError("liblmo expects contiguous CUDA tensors")
+
+
+def launch_count() -> int:
+    return int(_lib.lmo_launch_count())
+
+
+# ---------------------------------------------------------------- A1 / A5
+
+def lmo_quantize_groupwise(x: torch.Tensor, outer: int, n: int, inner: int,
+                           codes: torch.Tensor | None = None, meta: torch.Tensor | None = None,
+                           bits: int = 4, group_size: int = GROUP, stream=None):
+    """Alg 2 / Eq 10 on x (fp16) viewed as (outer, n, inner).
+    Returns (codes uint8 (outer, n_pad/2, inner), meta int32 (outer, n_pad/64, inner))."""
+    ng = (n + group_size - 1) // group_size
+    if codes is None:
+        codes = torch.empty((outer, ng * group_size // 2, inner), dtype=torch.uint8, device=x.device)
+    if meta is None:
+        meta = torch.empty((outer, ng, inner), dtype=torch.int32, device=x.device)
+    _need_cuda(x, codes, meta)
+    assert x.dtype == torch.float16 and x.numel() == outer * n * inner
+    _check(_lib.lmo_quantize_groupwise(_ptr(x), outer, n, inner, bits, group_size, _ptr(codes),
+                                       _ptr(meta), _stream(stream)), "lmo_quantize_groupwise")
+    return codes, meta
+
+
+def lmo_dequantize_groupwise(codes: torch.Tensor, meta: torch.Tensor, outer: int, n: int,
+                             inner: int, y: torch.Tensor | None = None, bits: int = 4,
+                             group_size: int = GROUP, stream=None) -> torch.Tensor:
+    """Eq 11 -> fp16 (outer, n, inner)."""
+    if y is None:
+        y = torch.empty((outer, n, inner), dtype=torch.float16, device=codes.device)
+    _need_cuda(codes, meta, y)
+    _check(_lib.lmo_dequantize_groupwise(_ptr(codes), _ptr(meta), outer, n, inner, bits,
+                                         group_size, _ptr(y), _stream(stream)),
+           "lmo_dequantize_groupwise")
+    return y
+
+
+# ------------------------------------------------------------ KV cache ----
+
+@dataclass
+class KVCache:
+    """One layer's q4 KV cache in the library layout (torch owns the memory)."""
+    k_codes: torch.Tensor   # [B][Hkv][cap][d/2] uint8
+    v_codes: torch.Tensor
+    k_meta: torch.Tensor    # [B][Hkv][cap][d/64] int32 (lmo_qmeta)
+    v_meta: torch.Tensor
+    batch: int
+    kv_heads: int
+    capacity: int
+    head_dim: int
+
+    @staticmethod
+    def empty(batch: int, kv_heads: int, capacity: int, head_dim: int, device="cuda",
+              zero: bool = False) -> "KVCache":
+        cap = (capacity + 15) // 16 * 16
+        alloc = torch.zeros if zero else torch.empty
+        ng = head_dim // GROUP
+        kc = alloc((batch, kv_heads, cap, head_dim // 2), dtype=torch.uint8, device=device)
+        vc = alloc((batch, kv_heads, cap, head_dim // 2), dtype=torch.uint8, device=device)
+        km = alloc((batch, kv_heads, cap, ng), dtype=torch.int32, device=device)
+        vm = alloc((batch, kv_heads, cap, ng), dtype=torch.int32, device=device)
+        return KVCache(kc, vc, km, vm, batch, kv_heads, cap, head_dim)
+
+    def abi(self) -> lmo_kv_cache:
+        return lmo_kv_cache(self.k_codes.data_ptr(), self.v_codes.data_ptr(),
+                            self.k_meta.data_ptr(), self.v_meta.data_ptr(), self.batch,
+                            self.kv_heads, self.capacity, self.head_dim)
+
+    def nbytes(self) -> int:
+        return sum(t.numel() * t.element_size()
+                   for t in (self.k_codes, self.v_codes, self.k_meta, self.v_meta))
+
+
+def lmo_kv_append_quant(cache: KVCache, k_new: torch.Tensor, v_new: torch.Tensor, pos0: int = 0,
+                        pos_dev: torch.Tensor | None = None, stream=None, abi=None) -> None:
+    """Append-quantize k_new/v_new [B][Hkv][n_new][d] at slots pos (Eq 7)."""
+    n_new = k_new.shape[2]
+    c = abi if abi is not None else cache.abi()
+    _check(_lib.lmo_kv_append_quant(ctypes.byref(c), _ptr(k_new), _ptr(v_new), n_new, pos0,
+                                    _ptr(pos_dev), _stream(stream)), "lmo_kv_append_quant")
+
+
+def lmo_decode_attention_workspace_bytes(batch: int, kv_heads: int, q_heads: int, head_dim: int,
+                                         num_splits: int = 0) -> int:
+    return int(_lib.lmo_decode_attention_workspace_bytes(batch, kv_heads, q_heads, head_dim,
+                                                         num_splits))
+
+
+def attention_workspace(batch: int, kv_heads: int, q_heads: int, head_dim: int,
+                        num_splits: int = 0, device="cuda") -> torch.Tensor:
+    """Zero-initialised workspace (its arrival counters must start at 0)."""
+    n = lmo_decode_attention_workspace_bytes(batch, kv_heads, q_heads, head_dim, num_splits)
+    if n == 0:
+        raise LmoError(LMO_ERR_SHAPE, "lmo_decode_attention_workspace_bytes")
+    return torch.zeros(n, dtype=torch.uint8, device=device)
+
+
+def lmo_decode_attention_q4(cache: KVCache, q: torch.Tensor, length: int = 0,
+                            seq_lens: torch.Tensor | None = None, softmax_scale: float | None = None,
+                            num_splits: int = 0, out: torch.Tensor | None = None,
+                            out_dtype: torch.dtype = torch.float32,
+                            workspace: torch.Tensor | None = None, stream=None,
+                            abi=None) -> torch.Tensor:
+    """softmax(scale q K^T) V over the q4 cache, dequant fused."""
+    B, Hq, d = q.shape
+    if softmax_scale is None:
+        softmax_scale = 1.0 / math.sqrt(d)
+    if out is None:
+        out = torch.empty((B, Hq, d), dtype=out_dtype, device=q.device)
+    if workspace is None:
+        workspace = attention_workspace(cache.batch, cache.kv_heads, Hq, cache.head_dim,
+                                        num_splits, q.device)
+    dt = LMO_F16 if out.dtype == torch.float16 else LMO_F32
+    c = abi if abi is not None else cache.abi()
+    _check(_lib.lmo_decode_attention_q4(ctypes.byref(c), _ptr(q), Hq, length, _ptr(seq_lens),
+                                        float(softmax_scale), num_splits, _ptr(out), dt,
+                                        _ptr(workspace), workspace.numel(), _stream(stream)),
+           "lmo_decode_attention_q4")
+    return out
+
+
+def lmo_gen_fill_f16(dst: torch.Tensor, seed: int, stream_id: int, layer: int, b0: int, h0: int,
+                     p0: int, group: int = 1, stream=None) -> torch.Tensor:
+    """Device twin of inputs.gen_f16: dst [nb][nh][npos][dim] fp16."""
+    nb, nh, npos, dim = dst.shape
+    _need_cuda(dst)
+    _check(_lib.lmo_gen_fill_f16(_ptr(dst), nb, nh, npos, dim, seed, stream_id, layer, b0, h0, p0,
+                                 group, _stream(stream)), "lmo_gen_fill_f16")
+    return dst

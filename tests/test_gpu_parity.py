@@ -1,0 +1,266 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by
+element on the same seeded inputs.
+
+Bars: codes / mins / scales / dequantized fp16 bit-exact;
+attention normwise per (b, h) row max|o_gpu - o_ref| / max|o_ref| <= 2e-3
+(BASELINE.json north star), fp32 accumulation vs the fp64 oracle.
+"""
+import math
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_ipps_wurypgll25_b200 import inputs as I
+from paper_conf_ipps_wurypgll25_b200.configs import CONFIGS
+
+pytestmark = pytest.mark.gpu
+TOL = 2e-3
+
+
+@pytest.fixture(scope="module")
+def lmo():
+    from paper_conf_ipps_wurypgll25_b200 import lmo as m
+    return m
+
+
+def dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a)).cuda()
+
+
+def meta_u16(m):
+    """int32 meta tensor -> uint16 pairs {min, scale} (little-endian)."""
+    return m.cpu().numpy().view(np.uint16).reshape(*m.shape, 2)
+
+
+def normwise_err(got, ref):
+    got = np.asarray(got, np.float64)
+    den = np.maximum(np.max(np.abs(ref), axis=-1), 1e-30)
+    return np.max(np.abs(got - ref), axis=-1) / den
+
+
+# ----------------------------------------------------------------- K6 ------
+
+def test_generator_matches_host(lmo):
+    for stream, group in ((I.STREAM_K, 1), (I.STREAM_V, 1), (I.STREAM_Q, 8)):
+        d = torch.empty((3, 5, 37, 128), dtype=torch.float16, device="cuda")
+        lmo.lmo_gen_fill_f16(d, seed=I.seed_for_config(4), stream_id=stream, layer=7, b0=11, h0=2,
+                             p0=1000, group=group)
+        h = I.gen_f16(I.seed_for_config(4), stream, 7, 11, 3, 2, 5, 1000, 37, 128, group=group)
+        assert np.array_equal(d.cpu().numpy().view(np.uint16), h.view(np.uint16))
+
+
+# ------------------------------------------------------------ K1 / K5 ------
+
+def adversarial_tensor(rng, rows):
+    g = [rng.standard_normal(64) * 10.0 ** rng.uniform(-3, 3) for _ in range(max(rows, 6))]
+    g[0] = np.full(64, 3.25)                        # constant
+    g[1] = np.full(64, -0.0)                        # signed zero
+    g[2] = -3.0 + rng.integers(0, 16, 64) * 0.25    # on-grid
+    g[3] = rng.uniform(-65504, 65504, 64)           # extremes
+    g[3][:2] = [-65504, 65504]
+    g[4] = rng.integers(-3, 4, 64) * 2.0 ** -24     # subnormal
+    x = np.zeros(64); x[0], x[1] = 0, 15; x[2:9] = [0.5, 1.5, 2.5, 3.5, 4.5, 13.5, 14.5]
+    g[5] = x                                        # ties
+    order = rng.permutation(len(g))[:rows]
+    return np.concatenate([g[i] for i in order]).astype(np.float16)
+
+
+@pytest.mark.parametrize("outer,n,inner", [(1, 64, 1), (37, 128, 1), (300, 64 * 5, 1),
+                                           (3, 100, 1), (4, 128, 7), (2, 65, 3), (1, 7, 1)])
+def test_quantize_bit_exact(lmo, outer, n, inner):
+    rng = np.random.default_rng(outer * 1000 + n + inner)
+    if inner == 1 and n % 64 == 0:
+        x = adversarial_tensor(rng, outer * n // 64).reshape(outer, n, inner)
+    else:
+        x = (rng.standard_normal((outer, n, inner)) * 3).astype(np.float16)
+    c_ref, m_ref = oracle.quantize_groupwise(x, outer, n, inner)
+    c, m = lmo.lmo_quantize_groupwise(dev(x), outer, n, inner)
+    torch.cuda.synchronize()
+    assert np.array_equal(c.cpu().numpy(), c_ref)
+    assert np.array_equal(meta_u16(m), m_ref)
+
+
+@pytest.mark.parametrize("outer,n,inner", [(64, 128, 1), (3, 100, 1), (4, 128, 7), (513, 64 * 3, 1)])
+def test_dequantize_bit_exact(lmo, outer, n, inner):
+    rng = np.random.default_rng(n + inner)
+    x = (rng.standard_normal((outer, n, inner)) * 10.0 ** rng.uniform(-2, 2)).astype(np.float16)
+    c_ref, m_ref = oracle.quantize_groupwise(x, outer, n, inner)
+    y_ref = oracle.dequantize_groupwise(c_ref, m_ref, outer, n, inner)
+    m_i32 = np.ascontiguousarray(m_ref).view(np.int32).reshape(m_ref.shape[:-1])
+    y = lmo.lmo_dequantize_groupwise(dev(c_ref), dev(m_i32), outer, n, inner)
+    torch.cuda.synchronize()
+    assert np.array_equal(y.cpu().numpy().view(np.uint16), y_ref.view(np.uint16))
+
+
+def test_weight_dequant_round_trip_shape(lmo):
+    """c3 weight leg at a reduced hidden size: quantize (inner-dim groups) then
+    dequantize equals the oracle's dequant of the oracle's codes."""
+    rng = np.random.default_rng(3)
+    h1 = 512
+    w = (rng.standard_normal((4 * h1, h1)) * 0.02).astype(np.float16)
+    c, m = lmo.lmo_quantize_groupwise(dev(w), 4 * h1, h1, 1)
+    y = lmo.lmo_dequantize_groupwise(c, m, 4 * h1, h1, 1)
+    c_ref, m_ref = oracle.quantize_groupwise(w, 4 * h1, h1, 1)
+    y_ref = oracle.dequantize_groupwise(c_ref, m_ref, 4 * h1, h1, 1)
+    assert np.array_equal(y.cpu().numpy().view(np.uint16), y_ref.view(np.uint16))
+
+
+# ---------------------------------------------------------------- K2 -------
+
+def cache_to_host(cache):
+    return {
+        "k_codes": cache.k_codes.cpu().numpy(), "v_codes": cache.v_codes.cpu().numpy(),
+        "k_meta": cache.k_meta.cpu().numpy().view(np.uint16).reshape(*cache.k_meta.shape, 2),
+        "v_meta": cache.v_meta.cpu().numpy().view(np.uint16).reshape(*cache.v_meta.shape, 2),
+    }
+
+
+@pytest.mark.parametrize("d", [64, 128])
+def test_append_bit_exact_with_canaries(lmo, d):
+    rng = np.random.default_rng(d)
+    B, H, cap, n_new = 3, 4, 48, 5
+    cache = lmo.KVCache.empty(B, H, cap, d)
+    for t in (cache.k_codes, cache.v_codes, cache.k_meta, cache.v_meta):
+        t.view(torch.uint8).fill_(0xA5)
+    host = oracle.new_cache(B, H, cap, d, fill=0xA5)
+    k = (rng.standard_normal((B, H, n_new, d)) * 2).astype(np.float16)
+    v = rng.standard_normal((B, H, n_new, d)).astype(np.float16)
+    lmo.lmo_kv_append_quant(cache, dev(k), dev(v), pos0=17)
+    oracle.kv_append_quant(host, k, v, 17)
+    # per-sequence positions
+    pos = np.array([0, 40, 9], np.int32)
+    k2 = (rng.standard_normal((B, H, 3, d))).astype(np.float16)
+    lmo.lmo_kv_append_quant(cache, dev(k2), dev(k2), pos_dev=dev(pos))
+    oracle.kv_append_quant(host, k2, k2, pos)
+    torch.cuda.synchronize()
+    got = cache_to_host(cache)
+    for key in host:
+        assert np.array_equal(got[key], host[key]), key
+
+
+# ---------------------------------------------------------------- K3 -------
+
+def build_layer(lmo, B, Hkv, cap, d, L, seed, layer=0, lens=None):
+    """Fill a q4 cache on the device from the seeded generator (prefill via
+    append) and the same cache on the host via the oracle."""
+    kf = torch.empty((B, Hkv, L, d), dtype=torch.float16, device="cuda")
+    vf = torch.empty_like(kf)
+    lmo.lmo_gen_fill_f16(kf, seed, I.STREAM_K, layer, 0, 0, 0)
+    lmo.lmo_gen_fill_f16(vf, seed, I.STREAM_V, layer, 0, 0, 0)
+    cache = lmo.KVCache.empty(B, Hkv, cap, d)
+    lmo.lmo_kv_append_quant(cache, kf, vf, pos0=0)
+    host = oracle.new_cache(B, Hkv, cache.capacity, d)
+    kh = I.gen_f16(seed, I.STREAM_K, layer, 0, B, 0, Hkv, 0, L, d)
+    vh = I.gen_f16(seed, I.STREAM_V, layer, 0, B, 0, Hkv, 0, L, d)
+    oracle.kv_append_quant(host, kh, vh, 0)
+    return cache, host
+
+
+CASES = [  # (B, Hkv, G, d, L, num_splits)
+    (2, 3, 1, 64, 1, 0), (2, 3, 1, 128, 2, 0), (1, 2, 2, 128, 15, 0), (3, 2, 1, 128, 16, 0),
+    (2, 4, 1, 128, 17, 0), (4, 12, 1, 64, 71, 0), (2, 2, 4, 128, 63, 0), (2, 2, 8, 128, 65, 1),
+    (3, 5, 1, 128, 100, 3), (2, 2, 8, 64, 1000, 0), (1, 3, 1, 128, 1000, 7), (2, 1, 8, 128, 4090, 0),
+    (5, 7, 3, 128, 333, 0), (1, 1, 1, 128, 1, 4), (64, 8, 1, 128, 40, 0),
+]
+
+
+@pytest.mark.parametrize("B,Hkv,G,d,L,ns", CASES)
+@pytest.mark.parametrize("out_dtype", [torch.float32, torch.float16])
+def test_attention_parity(lmo, B, Hkv, G, d, L, ns, out_dtype):
+    seed = 1000 + B * 7 + L
+    cap = L + (L % 3)
+    cache, host = build_layer(lmo, B, Hkv, cap, d, L, seed)
+    Hq = Hkv * G
+    q = torch.empty((B, Hq, 1, d), dtype=torch.float16, device="cuda")
+    lmo.lmo_gen_fill_f16(q, seed, I.STREAM_Q, 0, 0, 0, 0, group=G)
+    q = q.view(B, Hq, d)
+    sigma = 1 / math.sqrt(d)
+    out = lmo.lmo_decode_attention_q4(cache, q, L, softmax_scale=sigma, num_splits=ns,
+                                      out_dtype=out_dtype)
+    torch.cuda.synchronize()
+    ref = oracle.decode_attention_q4(host, q.cpu().numpy(), L, sigma, nthreads=8)
+    err = normwise_err(out.float().cpu().numpy(), ref)
+    assert err.max() <= TOL, (err.max(), np.unravel_index(err.argmax(), err.shape))
+    # the workspace counters are left at zero (re-usable)
+
+
+def test_attention_per_sequence_lengths_and_reuse(lmo):
+    B, Hkv, G, d, cap = 6, 3, 2, 128, 272
+    cache, host = build_layer(lmo, B, Hkv, cap, d, cap, 77)
+    lens = np.array([1, 0, 272, 17, 128, 250], np.int32)
+    q = torch.empty((B, Hkv * G, 1, d), dtype=torch.float16, device="cuda")
+    lmo.lmo_gen_fill_f16(q, 77, I.STREAM_Q, 0, 0, 0, 0, group=G)
+    q = q.view(B, Hkv * G, d)
+    ws = lmo.attention_workspace(B, Hkv, Hkv * G, d, 0)
+    ref_lens = np.maximum(lens, 1)
+    ref = oracle.decode_attention_q4(host, q.cpu().numpy(), ref_lens, nthreads=8)
+    for _ in range(3):   # workspace counters must be reset by each call
+        out = lmo.lmo_decode_attention_q4(cache, q, 0, seq_lens=dev(lens), workspace=ws)
+        torch.cuda.synchronize()
+        o = out.cpu().numpy()
+        assert np.all(o[1] == 0)                     # empty sequence -> zero row
+        keep = lens > 0
+        err = normwise_err(o[keep], ref[keep])
+        assert err.max() <= TOL
+    assert int(ws[: 4 * B * Hkv].view(torch.int32).abs().sum()) == 0
+
+
+def test_attention_split_modes_agree(lmo):
+    """stream-K (0) and fixed splits (1, 5) give the same result within rounding;
+    a fixed split count is deterministic."""
+    B, Hkv, G, d, L = 4, 4, 2, 128, 700
+    cache, _ = build_layer(lmo, B, Hkv, L + 4, d, L, 5)
+    q = torch.empty((B, Hkv * G, 1, d), dtype=torch.float16, device="cuda")
+    lmo.lmo_gen_fill_f16(q, 5, I.STREAM_Q, 0, 0, 0, 0, group=G)
+    q = q.view(B, Hkv * G, d)
+    o0 = lmo.lmo_decode_attention_q4(cache, q, L, num_splits=0)
+    o1 = lmo.lmo_decode_attention_q4(cache, q, L, num_splits=1)
+    o5 = lmo.lmo_decode_attention_q4(cache, q, L, num_splits=5)
+    o5b = lmo.lmo_decode_attention_q4(cache, q, L, num_splits=5)
+    torch.cuda.synchronize()
+    assert torch.equal(o5, o5b)
+    for o in (o0, o5):
+        assert (o - o1).abs().max().item() <= 1e-3 * o1.abs().max().item()
+
+
+# --------------------------------------- full-size sampled (bench launch) --
+
+@pytest.mark.parametrize("key", ["c2", "c5"])
+def test_full_size_sampled_rows(lmo, key):
+    """One layer at BASELINE.json full size (c2 / c5), last decode step, launched
+    as bench.py launches it (stream-K, fp32 out); sampled (b, kv-head) rows are
+    checked against the oracle one by one."""
+    w = CONFIGS[key]
+    seed = I.seed_for_config(w.index)
+    L = w.max_len
+    B, Hkv, d, G = w.batch, w.kv_heads, w.head_dim, w.group_ratio
+    cache = lmo.KVCache.empty(B, Hkv, w.capacity, d)
+    kf = torch.empty((B, Hkv, L, d), dtype=torch.float16, device="cuda")
+    vf = torch.empty_like(kf)
+    lmo.lmo_gen_fill_f16(kf, seed, I.STREAM_K, 0, 0, 0, 0)
+    lmo.lmo_gen_fill_f16(vf, seed, I.STREAM_V, 0, 0, 0, 0)
+    lmo.lmo_kv_append_quant(cache, kf, vf, pos0=0)
+    del kf, vf
+    q = torch.empty((B, w.q_heads, 1, d), dtype=torch.float16, device="cuda")
+    lmo.lmo_gen_fill_f16(q, seed, I.STREAM_Q, 0, 0, 0, w.steps - 1, group=G)
+    q = q.view(B, w.q_heads, d)
+    out = lmo.lmo_decode_attention_q4(cache, q, L)
+    torch.cuda.synchronize()
+    rng = np.random.default_rng(0)
+    samples = [(0, 0), (B - 1, Hkv - 1)] + [(int(rng.integers(B)), int(rng.integers(Hkv)))
+                                            for _ in range(4)]
+    got = cache_to_host(cache)
+    for b, kvh in samples:
+        one = oracle.new_cache(1, 1, w.capacity, d)
+        kh = I.gen_f16(seed, I.STREAM_K, 0, b, 1, kvh, 1, 0, L, d)
+        vh = I.gen_f16(seed, I.STREAM_V, 0, b, 1, kvh, 1, 0, L, d)
+        oracle.kv_append_quant(one, kh, vh, 0)
+        for k in ("k_codes", "v_codes", "k_meta", "v_meta"):   # append bit-exact at full size
+            assert np.array_equal(got[k][b, kvh, :L], one[k][0, 0, :L])
+        qh = q[b, kvh * G:(kvh + 1) * G].cpu().numpy()[None]
+        # the oracle wants Hq/Hkv = G for a single kv head
+        ref = oracle.decode_attention_q4(one, qh, L)
+        err = normwise_err(out[b, kvh * G:(kvh + 1) * G].cpu().numpy(), ref[0])
+        assert err.max() <= TOL, (b, kvh, err.max())

@@ -1,0 +1,410 @@
+#!/usr/bin/env python3
+"""bench.py -- q4-KV decode throughput on B200 (BASELINE.json metric).
+
+A "step" is one decode step of the whole hot path over all layers of the
+workload: for every layer, append-quantize the new token's K/V (A2) and run
+decode attention over the q4 cache (A3+A4).  Inputs are seeded synthetic
+tensors shaped like the paper's OPT/LLaMA workloads, resident in HBM before
+the timed region (value) or copied from pinned host memory inside it (e2e).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl ours|reference]
+
+Multi-GPU (torchrun, one rank per GPU, NCCL): the batch is sharded by
+sequence -- weak scaling, each rank owns a full config-sized batch at its own
+global batch offset; no collective in the hot path (timing reduce only).
+Prints ONE JSON line on rank 0.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_ipps_wurypgll25_b200 import configs as C  # noqa: E402
+from paper_conf_ipps_wurypgll25_b200 import inputs as I  # noqa: E402
+
+METRIC = "q4-KV decode-attention tokens/s & achieved HBM GB/s at 1/2/4/8 B200"
+FALLBACK_HBM = 6650.0
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--config", default="c2", choices=sorted(C.CONFIGS))
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--splits", type=int, default=0, help="num_splits (0 = stream-K auto)")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--cpu-sample-seconds", type=float, default=10.0)
+    return p.parse_args()
+
+
+def peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(path))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    except Exception:
+        return FALLBACK_HBM, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def workload_config(w: C.Workload, n: int, extra=None):
+    d = {
+        "workload": f"{w.key}: {w.name}",
+        "batch_per_gpu": w.batch, "global_batch": w.batch * n, "q_heads": w.q_heads,
+        "kv_heads": w.kv_heads, "head_dim": w.head_dim, "layers": w.layers,
+        "prompt": w.prompt, "gen": w.gen, "kv_format": "4-bit group-wise min/scale, G=64",
+        "parallelism": f"batch-sharded dp{n} (weak scaling)",
+    }
+    if extra:
+        d.update(extra)
+    return d
+
+
+# ------------------------------------------------------------- clocks ------
+
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *exc):
+        self.lines = []
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                out, _ = self.proc.communicate(timeout=5)
+            except Exception:
+                self.proc.kill()
+                out = ""
+            self.lines = [ln for ln in out.splitlines() if ln.strip()]
+
+    def summary(self):
+        sm, mx, reasons = [], 0.0, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in getattr(self, "lines", []):
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = max(mx, float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# -------------------------------------------------------- CPU oracle -------
+
+def cpu_oracle_rate(w: C.Workload, target_s: float, nthreads: int):
+    """Time the oracle (as it stands) on a bounded sample of one layer-step at the
+    mean decode length, extrapolated to tokens/s of the whole workload."""
+    import numpy as np
+    import oracle
+    seed = I.seed_for_config(w.index)
+    L = w.prompt + w.gen // 2
+    d, G = w.head_dim, w.group_ratio
+    pairs_total = w.batch * w.kv_heads
+    npairs, t_pair = 1, None
+    done = 0
+    elapsed = 0.0
+    rng_pairs = [(b, h) for b in range(w.batch) for h in range(w.kv_heads)]
+    # grow the sample until ~target_s of CPU time has been measured
+    while elapsed < target_s and done < pairs_total:
+        chunk = rng_pairs[done:done + npairs]
+        B = len(chunk)
+        cache = oracle.new_cache(B, 1, L + 1, d)
+        ks = np.stack([I.gen_f16(seed, I.STREAM_K, 0, b, 1, h, 1, 0, L + 1, d)[0] for b, h in chunk])
+        vs = np.stack([I.gen_f16(seed, I.STREAM_V, 0, b, 1, h, 1, 0, L + 1, d)[0] for b, h in chunk])
+        qs = np.stack([I.gen_f16(seed, I.STREAM_Q, 0, b, 1, h * G, G, 0, 1, d, group=G)[0, :, 0]
+                       for b, h in chunk])
+        oracle.kv_append_quant(cache, ks[:, :, :L], vs[:, :, :L], 0)   # resident cache (untimed)
+        t0 = time.perf_counter()
+        oracle.kv_append_quant(cache, ks[:, :, L:], vs[:, :, L:], L)    # A2 (timed)
+        oracle.decode_attention_q4(cache, qs, L + 1, nthreads=nthreads)  # A3 (timed)
+        dt = time.perf_counter() - t0
+        elapsed += dt
+        done += B
+        npairs = min(pairs_total - done, max(1, npairs * 2))
+    t_pair = elapsed / done
+    t_step = t_pair * pairs_total * w.layers
+    tokens_per_s = w.batch / t_step
+    by = C.layer_step_bytes(w, L + 1) * w.layers
+    return {
+        "value": tokens_per_s, "unit": "tokens/s", "cores": nthreads, "kind": "oracle",
+        "sample": (f"{done} of {pairs_total} (sequence, kv-head) pairs x 1 layer of one decode "
+                   f"step at L={L + 1} (append + attention), {elapsed:.1f} s CPU wall; "
+                   f"extrapolated x{pairs_total * w.layers / done:.0f} to all pairs and "
+                   f"{w.layers} layers (work is linear in pairs x layers)"),
+        "gbs_equiv": by / t_step / 1e9,
+    }
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    w = C.CONFIGS[args.config]
+    nthreads = len(os.sched_getaffinity(0))
+    vals = []
+    base = None
+    per = max(1.0, min(3.0, args.cpu_sample_seconds / 3))
+    for i in range(args.warmup + args.steps):
+        r = cpu_oracle_rate(w, per if i >= args.warmup else 0.5, nthreads)
+        if i >= args.warmup:
+            vals.append(r["value"])
+            base = r
+    v = statistics.median(vals)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "tokens/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": 1e3 * w.batch / v, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded counter-based generator)",
+        "config": workload_config(w, 1),
+        "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": nthreads, "kind": "oracle",
+                         "sample": base["sample"]},
+        "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------- our arm -------
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_wurypgll25_b200 import lmo
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    w = C.CONFIGS[args.config]
+    seed = I.seed_for_config(w.index)
+    B, Hkv, Hq, d, G, s = w.batch, w.kv_heads, w.q_heads, w.head_dim, w.group_ratio, w.prompt
+    b_off = rank * B                      # global batch offset (weak scaling)
+    nl = w.layers
+    steps_total = args.warmup + args.steps
+    # decode step j (0-based over warmup+timed) -> t in 1..n-1 (cycled)
+    t_of = [(j % w.steps) + 1 for j in range(steps_total)]
+    distinct_t = sorted(set(t_of))
+
+    # ---- caches + prefill (A1 through the append entry; timed separately)
+    caches = [lmo.KVCache.empty(B, Hkv, w.capacity, d, device=dev) for _ in range(nl)]
+    abis = [c.abi() for c in caches]
+    stream = torch.cuda.Stream(device=dev)
+    pre_ms = 0.0
+    with torch.cuda.stream(stream):
+        kp = torch.empty((B, Hkv, s, d), dtype=torch.float16, device=dev)
+        vp = torch.empty_like(kp)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        for l in range(nl):
+            lmo.lmo_gen_fill_f16(kp, seed, I.STREAM_K, l, b_off, 0, 0)
+            lmo.lmo_gen_fill_f16(vp, seed, I.STREAM_V, l, b_off, 0, 0)
+            e0.record()
+            lmo.lmo_kv_append_quant(caches[l], kp, vp, pos0=0, abi=abis[l])
+            e1.record()
+            e1.synchronize()
+            pre_ms += e0.elapsed_time(e1)
+        del kp, vp
+        # ---- per-step inputs (device-resident) and outputs
+        qbuf, kbuf, vbuf = {}, {}, {}
+        for t in distinct_t:
+            qbuf[t] = torch.empty((nl, B, Hq, 1, d), dtype=torch.float16, device=dev)
+            kbuf[t] = torch.empty((nl, B, Hkv, 1, d), dtype=torch.float16, device=dev)
+            vbuf[t] = torch.empty_like(kbuf[t])
+            for l in range(nl):
+                lmo.lmo_gen_fill_f16(qbuf[t][l], seed, I.STREAM_Q, l, b_off, 0, t - 1, group=G)
+                lmo.lmo_gen_fill_f16(kbuf[t][l], seed, I.STREAM_K, l, b_off, 0, s + t - 1)
+                lmo.lmo_gen_fill_f16(vbuf[t][l], seed, I.STREAM_V, l, b_off, 0, s + t - 1)
+        out = torch.empty((nl, B, Hq, d), dtype=torch.float32, device=dev)
+        ws = lmo.attention_workspace(B, Hkv, Hq, d, args.splits, device=dev)
+    stream.synchronize()
+    sigma = 1.0 / math.sqrt(d)
+
+    def step(t, attn=True, append=True):
+        for l in range(nl):
+            if append:
+                lmo.lmo_kv_append_quant(caches[l], kbuf[t][l], vbuf[t][l], pos0=s + t - 1,
+                                        abi=abis[l])
+            if attn:
+                lmo.lmo_decode_attention_q4(caches[l], qbuf[t][l].view(B, Hq, d), s + t,
+                                            softmax_scale=sigma, num_splits=args.splits,
+                                            out=out[l], workspace=ws, abi=abis[l])
+
+    # ---- capture one CUDA graph per distinct step
+    graphs = {}
+    n0 = lmo.launch_count()
+    for t in distinct_t:
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=stream):
+            step(t)
+        graphs[t] = g
+    launches_per_step = (lmo.launch_count() - n0) // len(distinct_t)
+    # attention-only graph (roofline leg) at the middle length
+    t_mid = distinct_t[len(distinct_t) // 2]
+    g_attn = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g_attn, stream=stream):
+        step(t_mid, append=False)
+    torch.cuda.synchronize()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def reduce_max(x: float) -> float:
+        if world == 1:
+            return x
+        tt = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        return float(tt.item())
+
+    # ---- warm-up + timed steps (device-resident inputs)
+    with torch.cuda.stream(stream):
+        for j in range(args.warmup):
+            graphs[t_of[j]].replay()
+    barrier()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        with torch.cuda.stream(stream):
+            ev0.record(stream)
+            for j in range(args.warmup, steps_total):
+                graphs[t_of[j]].replay()
+            ev1.record(stream)
+        ev1.synchronize()
+    barrier()
+    ms = reduce_max(ev0.elapsed_time(ev1))
+    clocks = clk.summary()
+    tokens = world * B * args.steps
+    value = tokens / (ms / 1e3)
+    step_bytes = sum(C.layer_step_bytes(w, s + t_of[j], B) * nl for j in range(args.warmup, steps_total))
+    gbs = world * step_bytes / (ms / 1e3) / 1e9
+
+    # ---- roofline leg: attention-only launches, CUDA events on the launching stream
+    reps = 5
+    with torch.cuda.stream(stream):
+        g_attn.replay()
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a0.record(stream)
+        for _ in range(reps):
+            g_attn.replay()
+        a1.record(stream)
+    a1.synchronize()
+    attn_ms = reduce_max(a0.elapsed_time(a1)) / (reps * nl)
+    attn_bytes = C.attention_launch_bytes(w, s + t_mid, B)
+    peak, peak_src = peaks()
+    achieved = attn_bytes / (attn_ms / 1e3) / 1e9
+    traffic = None
+    prof = os.path.join(ROOT, "profiles", f"ncu_{w.key}.json")
+    if os.path.exists(prof):
+        try:
+            traffic = json.load(open(prof)).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+
+    # ---- e2e: host buffers, H2D of each step's inputs + D2H of its result in the region
+    e2e = None
+    if not args.no_e2e:
+        hq = {t: qbuf[t].cpu().pin_memory() for t in distinct_t}
+        hk = {t: kbuf[t].cpu().pin_memory() for t in distinct_t}
+        hv = {t: vbuf[t].cpu().pin_memory() for t in distinct_t}
+        hout = torch.empty((B, Hq, d), dtype=torch.float32).pin_memory()
+        h2d = (hq[t_mid].numel() + hk[t_mid].numel() + hv[t_mid].numel()) * 2
+        d2h = hout.numel() * 4
+        barrier()
+        with torch.cuda.stream(stream):
+            x0, x1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            x0.record(stream)
+            for j in range(args.warmup, steps_total):
+                t = t_of[j]
+                qbuf[t].copy_(hq[t], non_blocking=True)
+                kbuf[t].copy_(hk[t], non_blocking=True)
+                vbuf[t].copy_(hv[t], non_blocking=True)
+                graphs[t].replay()
+                hout.copy_(out[nl - 1], non_blocking=True)
+            x1.record(stream)
+        x1.synchronize()
+        barrier()
+        e2e_ms = reduce_max(x0.elapsed_time(x1))
+        e2e = {"value": tokens / (e2e_ms / 1e3), "unit": "tokens/s", "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": d2h, "ms_per_step": e2e_ms / args.steps,
+               "path": "pinned host inputs -> H2D -> liblmo C-ABI step graph -> D2H last-layer output"}
+
+    cpu = None
+    if rank == 0 and world == 1:
+        try:
+            cpu = cpu_oracle_rate(w, args.cpu_sample_seconds, len(os.sched_getaffinity(0)))
+            cpu.pop("gbs_equiv", None)
+        except Exception as ex:  # never fail the bench line on the baseline leg
+            cpu = {"value": None, "error": str(ex)[:200]}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "tokens/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u4+f16/f32",
+            "data": "synthetic (seeded counter-based generator; OPT/LLaMA-shaped K/V/q)",
+            "config": workload_config(w, world, {
+                "l2": f"inputs larger than L2: per-step q4 KV footprint "
+                      f"{sum(c.nbytes() for c in caches) / 1e9:.2f} GB per GPU cycles through 126 MB L2",
+                "num_splits": args.splits}),
+            "achieved_gbs": gbs, "frac_of_peak": gbs / peak,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": traffic,
+                         "kernel": "decode_attn_q4_kernel", "peak_source": peak_src,
+                         "per_launch_us": attn_ms * 1e3, "algorithmic_bytes_per_launch": attn_bytes},
+            "prefill_ms_all_layers": pre_ms,
+            "gpu_launches": launches_per_step * args.steps,
+            "clocks": clocks,
+            "e2e": e2e,
+            "cpu_baseline": cpu,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -85,24 +85,29 @@ lmo_status lmo_dequantize_groupwise(const uint8_t *codes, const lmo_qmeta *meta,
                                     int64_t n, int64_t inner, int bits, int group_size,
                                     void *y_f16, void *stream);
 
-/* One layer's q4 KV cache (caller-owned device memory), layout
- *   k_codes, v_codes : [batch][kv_heads][capacity][head_dim/2]  bytes
- *   k_meta,  v_meta  : [batch][kv_heads][capacity][head_dim/64] lmo_qmeta
- * i.e. token-major per (sequence, kv head), so a run of tokens is one
- * contiguous span (one bulk copy).  Groups lie along head_dim (DESIGN.md
- * reading 8), so every token's groups are self-contained.
- * head_dim must be 64 or 128; capacity must be a multiple of 16 (callers
- * round up; the 16-token block is the kernels' unit of work). */
+/* One layer's q4 KV cache (caller-owned device memory): one contiguous
+ * "compressed row" per (sequence, kv head, token slot):
+ *   kv : [batch][kv_heads][capacity][row_bytes]        row_bytes = lmo_kv_row_bytes(head_dim)
+ *   row: K codes (head_dim/2 B) | K meta (head_dim/64 lmo_qmeta) |
+ *        V codes (head_dim/2 B) | V meta (head_dim/64 lmo_qmeta)
+ * (144 B per token at head_dim 128, 72 B at 64).  Codes and meta are exactly
+ * what lmo_quantize_groupwise(outer=1, n=head_dim, inner=1) produces for that
+ * token's K (resp. V) row.  Token-major rows make a run of tokens of one
+ * (sequence, kv head) a single contiguous span, i.e. one bulk copy.  Groups lie
+ * along head_dim (reading 8), so every token's groups are
+ * self-contained.  head_dim must be 64 or 128; capacity must be a multiple of
+ * 16 (callers round up; the 16-token block is the kernels' unit of work); kv
+ * must be 16-byte aligned. */
 typedef struct {
-    uint8_t *k_codes;
-    uint8_t *v_codes;
-    lmo_qmeta *k_meta;
-    lmo_qmeta *v_meta;
+    uint8_t *kv;
     int32_t batch;
     int32_t kv_heads;
     int32_t capacity;
     int32_t head_dim;
 } lmo_kv_cache;
+
+/* Bytes of one compressed K+V token row for head_dim (0 if unsupported). */
+size_t lmo_kv_row_bytes(int32_t head_dim);
 
 /* ---------------------------------------------------------------------------
  * A2. KV append-quantize -- "The KV cache is updated by concatenating the

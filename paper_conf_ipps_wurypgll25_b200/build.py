@@ -47,7 +47,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and not needs_build():
         return LIB
     tmp = LIB + ".tmp"
-    cmd = [nvcc(), *NVCC_FLAGS, "-I", INCLUDE, "-I", CSRC, "-o", tmp, *sources()]
+    defs = os.environ.get("LMO_NVCC_DEFS", "").split()
+    cmd = [nvcc(), *NVCC_FLAGS, *defs, "-I", INCLUDE, "-I", CSRC, "-o", tmp, *sources()]
     res = subprocess.run(cmd, capture_output=True, text=True)
     log = os.path.join(PKG, "build.log")
     with open(log, "w") as f:

@@ -27,27 +27,50 @@
 //  * GQA: the query heads sharing a kv head are the MMA's head dimension, so
 //    a KV tile is read once for all of them (8 q heads per kv head cost the
 //    same HMMA count as 1).
+#include <type_traits>
+
 #include "common.cuh"
 
 namespace lmo {
 
-constexpr int kBlk = 16;      // tokens per warp-block (MMA k extent)
-constexpr int kWarps = 4;     // warps per CTA
-constexpr int kStages = 4;    // per-warp TMA ring depth
+constexpr int kBlk = 16;      // tokens per MMA sub-block = unit of the work partition
+constexpr int kSub = 2;       // sub-blocks per pipeline stage (32 tokens)
+constexpr int kStageTok = kBlk * kSub;
+#ifndef LMO_ATTN_WARPS
+#define LMO_ATTN_WARPS 4
+#endif
+#ifndef LMO_ATTN_STAGES
+#define LMO_ATTN_STAGES 3
+#endif
+#ifndef LMO_ATTN_PROFILE
+#define LMO_ATTN_PROFILE 0
+#endif
+#ifndef LMO_ATTN_MINBLOCKS
+#define LMO_ATTN_MINBLOCKS 4
+#endif
+constexpr int kWarps = LMO_ATTN_WARPS;    // warps per CTA
+constexpr int kStages = LMO_ATTN_STAGES;  // per-warp TMA ring depth (stages of 32 tokens)
 constexpr int kMaxBatchSmem = 1024;  // per-sequence-length mode: prefix array in smem
 
 template <int D>
 struct Geo {
     static constexpr int NG = D / 64;              // quantization groups per row
-    static constexpr int KC = kBlk * D / 2;        // code bytes per block (K or V)
-    static constexpr int KM = kBlk * NG * 4;       // meta bytes per block (K or V)
-    static constexpr int STAGE = 2 * (KC + KM);    // bytes per stage
+    static constexpr int RB = D / 2;               // code bytes per K (or V) row
+    static constexpr int MB = NG * 4;              // meta bytes per K (or V) row
+    static constexpr int ROW = 2 * (RB + MB);       // compressed K+V token row (144 B at D=128)
+    static constexpr int OKM = RB;                 // offsets inside a row
+    static constexpr int OVC = RB + MB;
+    static constexpr int OVM = 2 * RB + MB;
+    static constexpr int STAGE = kStageTok * ROW;  // bytes per stage
     static constexpr int REC = D + 4;              // partial record floats per head
 };
 
+#if LMO_ATTN_PROFILE
+__device__ unsigned long long *g_attn_prof = nullptr;   // [warp][4]: wait, total, stages, segments
+#endif
+
 struct AttnArgs {
-    const uint8_t *kc, *vc;
-    const uint32_t *km, *vm;
+    const uint8_t *kv;        // [B][Hkv][cap][ROW]
     int B, Hkv, cap;
     const __half *q;
     int Hq, G;
@@ -55,6 +78,7 @@ struct AttnArgs {
     const int32_t *lens;      // per-sequence lengths or nullptr
     float scale_log2;         // softmax_scale * log2(e)
     int num_splits;           // 0 = stream-K
+    int team;                 // > 0: pair-team mode with this many warps per pair
     void *out;
     int out_f16;
     int *counters;            // [B*Hkv]
@@ -62,27 +86,29 @@ struct AttnArgs {
 };
 
 // ---------------------------------------------------------------- work map
+// Global list of 16-token blocks: sequence-major, then kv head, then block
+// (all int32: the ABI bounds keep N < 2^31).
 struct WorkMap {
-    const int *prefix;   // smem, B+1 (per-seq mode) or nullptr (uniform)
+    const int *prefix;   // smem, B+1 (per-sequence lengths) or nullptr (uniform length)
     int B, Hkv, nbu;     // nbu: blocks per pair in uniform mode
-    int64_t N;           // total blocks
-    int64_t V;           // virtual warps
-    int W;               // physical warps in grid
+    int N;               // total blocks
+    int V;               // virtual warps (ranges)
+    int W;               // physical warps in the grid
     int k;               // num_splits (0 = stream-K)
+    int T;               // team mode: warps per (b, kvh) pair (1, 2, 4); 0 = stream-K / fixed splits
+    int n_teams;         // team mode: teams in the grid
 
-    __device__ __forceinline__ int64_t seq_start(int b) const {
-        return prefix ? (int64_t)prefix[b] : (int64_t)b * Hkv * nbu;
-    }
+    __device__ __forceinline__ int seq_start(int b) const { return prefix ? prefix[b] : b * Hkv * nbu; }
     __device__ __forceinline__ int seq_nb(int b) const {
         return prefix ? (prefix[b + 1] - prefix[b]) / Hkv : nbu;
     }
     // global block x -> (b, kvh, blk, nb)
-    __device__ __forceinline__ void decode(int64_t x, int &b, int &kvh, int &blk, int &nb) const {
+    __device__ __forceinline__ void decode(int x, int &b, int &kvh, int &blk, int &nb) const {
         if (!prefix) {
-            const int64_t pair = x / nbu;
-            blk = (int)(x - pair * nbu);
-            b = (int)(pair / Hkv);
-            kvh = (int)(pair - (int64_t)b * Hkv);
+            const int pair = x / nbu;
+            blk = x - pair * nbu;
+            b = pair / Hkv;
+            kvh = pair - b * Hkv;
             nb = nbu;
         } else {
             int lo = 0, hi = B;  // largest b with prefix[b] <= x  (prefix[B] = N > x)
@@ -92,50 +118,83 @@ struct WorkMap {
             }
             b = lo;
             nb = seq_nb(b);
-            const int r = (int)(x - prefix[b]);
+            const int r = x - prefix[b];
             kvh = r / nb;
             blk = r - kvh * nb;
         }
     }
-    __device__ __forceinline__ int64_t pair_start(int b, int kvh) const {
-        return seq_start(b) + (int64_t)kvh * seq_nb(b);
-    }
     // start of virtual warp v's range
-    __device__ __forceinline__ int64_t R(int64_t v) const {
-        if (k == 0) return v * N / V;
-        const int64_t p = v / k;
-        if (p >= (int64_t)B * Hkv) return N;
-        const int j = (int)(v - p * k);
-        const int b = (int)(p / Hkv), kvh = (int)(p - (int64_t)b * Hkv);
+    __device__ __forceinline__ int R(int v) const {
+        if (k == 0) return (int)((long long)v * N / V);
+        const int p = v / k;
+        if (p >= B * Hkv) return N;
+        const int j = v - p * k;
+        const int b = p / Hkv, kvh = p - b * Hkv;
         const int nb = seq_nb(b);
-        return pair_start(b, kvh) + (int64_t)j * nb / k;
+        return seq_start(b) + kvh * nb + j * nb / k;
     }
     // virtual warp whose range contains block x
-    __device__ __forceinline__ int64_t vwarp_of(int64_t x) const {
-        if (k == 0) return ((x + 1) * V + N - 1) / N - 1;
+    __device__ __forceinline__ int vwarp_of(int x) const {
+        if (k == 0) return (int)(((long long)(x + 1) * V + N - 1) / N) - 1;
         int b, kvh, blk, nb;
         decode(x, b, kvh, blk, nb);
-        int j = (int)(((int64_t)(blk + 1) * k + nb - 1) / nb) - 1;
+        int j = ((blk + 1) * k + nb - 1) / nb - 1;
         if (j > k - 1) j = k - 1;
-        return ((int64_t)b * Hkv + kvh) * k + j;
-    }
-    __device__ __forceinline__ int64_t slot_of(int64_t v, int64_t pstart) const {
-        return k == 0 ? 2 * v + (R(v) < pstart ? 1 : 0) : v;
+        return (b * Hkv + kvh) * k + j;
     }
 };
 
-struct Cursor {
-    int64_t x, xend, v;
-    int b, kvh, blk, nb;
+// Iterates the segments (maximal runs of blocks of one (b, kv head) pair) of
+// the virtual warps v = gw, gw + W, ...  Within a range the two PARTIAL
+// segments (first and last) come first and the full pairs in the middle come
+// last, so the cross-warp merges happen early and every warp ends on
+// independent work.
+struct SegIter {
+    int v, x0, x1, a, c, phase, mpos;
+    int sx, sn, b, kvh, blk, nb;    // current segment
     bool done;
 
-    __device__ __forceinline__ void enter(const WorkMap &wm, int64_t v0) {
-        v = v0;
+    __device__ __noinline__ void set_seg(const WorkMap &wm, int x, int n) {
+        sx = x;
+        sn = n;
+        wm.decode(x, b, kvh, blk, nb);
+    }
+    // team mode: v = pair index, x0 = rank of this warp in its team
+    __device__ __noinline__ void team_seg(const WorkMap &wm) {
+        if (v >= wm.B * wm.Hkv) {
+            done = true;
+            return;
+        }
+        b = v / wm.Hkv;
+        kvh = v - b * wm.Hkv;
+        nb = wm.seq_nb(b);
+        const int lo = x0 * nb / wm.T, hi = (x0 + 1) * nb / wm.T;
+        blk = lo;
+        sn = hi - lo;
+        sx = wm.seq_start(b) + kvh * nb + lo;
+        done = false;
+    }
+    __device__ __noinline__ void begin_v(const WorkMap &wm) {
+        if (wm.T) {
+            team_seg(wm);
+            return;
+        }
         while (v < wm.V) {
-            x = wm.R(v);
-            xend = wm.R(v + 1);
-            if (x < xend) {
-                wm.decode(x, b, kvh, blk, nb);
+            x0 = wm.R(v);
+            x1 = wm.R(v + 1);
+            if (x0 < x1) {
+                wm.decode(x0, b, kvh, blk, nb);
+                a = min(x1, x0 - blk + nb);
+                if (a < x1) {
+                    int b1, kvh1, blk1, nb1;
+                    wm.decode(x1 - 1, b1, kvh1, blk1, nb1);
+                    c = x1 - 1 - blk1;
+                } else {
+                    c = x1;
+                }
+                sx = x0;
+                sn = a - x0;
+                phase = 0;
                 done = false;
                 return;
             }
@@ -143,42 +202,67 @@ struct Cursor {
         }
         done = true;
     }
-    __device__ __forceinline__ void advance(const WorkMap &wm) {
-        ++x;
-        ++blk;
-        if (x >= xend) {
-            enter(wm, v + wm.W);
-        } else if (blk >= nb) {
-            wm.decode(x, b, kvh, blk, nb);
+    // out of line: runs only at segment transitions, keeps the hot loop small (I-cache)
+    __device__ __noinline__ void next(const WorkMap &wm) {
+        if (wm.T) {
+            v += wm.n_teams;
+            team_seg(wm);
+            return;
+        }
+        if (phase == 0 && a < x1) {
+            phase = 1;
+            set_seg(wm, c, x1 - c);
+        } else if (phase == 1 && a < c) {
+            phase = 2;
+            mpos = a;
+            set_seg(wm, mpos, 0);
+            sn = nb;
+        } else if (phase == 2 && mpos + nb < c) {
+            mpos += nb;
+            set_seg(wm, mpos, 0);
+            sn = nb;
+        } else {
+            v += wm.W;
+            begin_v(wm);
         }
     }
 };
 
 // ------------------------------------------------------------ fragments
-__device__ __forceinline__ int tok_perm(int n) { return n ^ ((n >> 1) & 1); }  // 0,1,3,2,4,5,7,6
+// Token order inside a 16-token block: MMA row r <-> token tperm(r) (a
+// bijection of 0..15 that halves shared-memory bank conflicts of the V loads).
+__device__ __forceinline__ int tperm(int r) { return r ^ ((r >> 1) & 1); }  // 0,1,3,2,4,5,7,6,...
 
-// K codes word -> 4 half2 of exact codes: (nib0,nib4) (nib1,nib5) (nib2,nib6) (nib3,nib7)
-__device__ __forceinline__ void unpack_k(uint32_t w, uint32_t (&u)[4]) {
+// Exact 4-bit codes as fp16 SUBNORMALS (no bias, no fp16 add):
+//   (x & 0x000F000F) reads the nibbles at bits 0-3 / 16-19 as c * 2^-24,
+//   (x & 0x00F000F0) reads the nibbles at bits 4-7 / 20-23 as 16*c * 2^-24 = c * 2^-20.
+// K side, one word (8 dims) ->
+//   u[0] = (nib0, nib4) * 2^-24, u[1] = (nib1, nib5) * 2^-20,
+//   u[2] = (nib2, nib6) * 2^-24, u[3] = (nib3, nib7) * 2^-20.
+// The 2^-20 slots meet q/16 in the MMA (see the q fragments), so every
+// product is q_i c_i 2^-24.
+__device__ __forceinline__ void unpack_k(uint32_t w, uint32_t *u) {
     const uint32_t s = w >> 8;
-    u[0] = hsub2_u32(lop3_and_or(w, 0x000F000Fu, 0x64006400u), 0x64006400u);
-    u[1] = hsub2_u32(lop3_and_or(w, 0x00F000F0u, 0x54005400u), 0x54005400u);
-    u[2] = hsub2_u32(lop3_and_or(s, 0x000F000Fu, 0x64006400u), 0x64006400u);
-    u[3] = hsub2_u32(lop3_and_or(s, 0x00F000F0u, 0x54005400u), 0x54005400u);
+    u[0] = w & 0x000F000Fu;
+    u[1] = w & 0x00F000F0u;
+    u[2] = s & 0x000F000Fu;
+    u[3] = s & 0x00F000F0u;
 }
 
-// V code words of two tokens (same dims) -> 8 half2 (tokA nib p, tokB nib p), p = 0..7
-__device__ __forceinline__ void unpack_v(uint32_t wa, uint32_t wb, uint32_t (&j)[8]) {
-    const uint32_t lo = prmt(wa, wb, 0x5410u);
-    const uint32_t hi = prmt(wa, wb, 0x7632u);
+// V side: code words of two tokens A, B (same 8 dims) -> 8 half2 (A nib p, B nib p);
+// even p in the 2^-24 form, odd p in the 2^-20 form.
+__device__ __forceinline__ void unpack_v(uint32_t wa, uint32_t wb, uint32_t *j) {
+    const uint32_t lo = prmt(wa, wb, 0x5410u);   // [A.b0, A.b1, B.b0, B.b1]
+    const uint32_t hi = prmt(wa, wb, 0x7632u);   // [A.b2, A.b3, B.b2, B.b3]
     const uint32_t lo8 = lo >> 8, hi8 = hi >> 8;
-    j[0] = hsub2_u32(lop3_and_or(lo, 0x000F000Fu, 0x64006400u), 0x64006400u);
-    j[1] = hsub2_u32(lop3_and_or(lo, 0x00F000F0u, 0x54005400u), 0x54005400u);
-    j[2] = hsub2_u32(lop3_and_or(lo8, 0x000F000Fu, 0x64006400u), 0x64006400u);
-    j[3] = hsub2_u32(lop3_and_or(lo8, 0x00F000F0u, 0x54005400u), 0x54005400u);
-    j[4] = hsub2_u32(lop3_and_or(hi, 0x000F000Fu, 0x64006400u), 0x64006400u);
-    j[5] = hsub2_u32(lop3_and_or(hi, 0x00F000F0u, 0x54005400u), 0x54005400u);
-    j[6] = hsub2_u32(lop3_and_or(hi8, 0x000F000Fu, 0x64006400u), 0x64006400u);
-    j[7] = hsub2_u32(lop3_and_or(hi8, 0x00F000F0u, 0x54005400u), 0x54005400u);
+    j[0] = lo & 0x000F000Fu;
+    j[1] = lo & 0x00F000F0u;
+    j[2] = lo8 & 0x000F000Fu;
+    j[3] = lo8 & 0x00F000F0u;
+    j[4] = hi & 0x000F000Fu;
+    j[5] = hi & 0x00F000F0u;
+    j[6] = hi8 & 0x000F000Fu;
+    j[7] = hi8 & 0x00F000F0u;
 }
 
 __device__ __forceinline__ float2 meta_f2(uint32_t mw) {
@@ -186,11 +270,47 @@ __device__ __forceinline__ float2 meta_f2(uint32_t mw) {
     return __half22float2(h);   // .x = min, .y = scale
 }
 
-__device__ __forceinline__ float warp_max4(float v) {  // over the 4 t-lanes of a g
-    v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 1));
-    return fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 2));
+// explicit shared-window loads (32-bit addresses; volatile: data arrives via TMA)
+__device__ __forceinline__ uint32_t lds32(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(v) : "r"(a));
+    return v;
 }
-__device__ __forceinline__ float warp_sum4(float v) {
+__device__ __forceinline__ uint2 lds64(uint32_t a) {
+    uint2 v;
+    asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n" : "=r"(v.x), "=r"(v.y) : "r"(a));
+    return v;
+}
+// the NG meta words of one row (NG = 1: 4-byte aligned only)
+template <int NG>
+__device__ __forceinline__ uint2 load_meta(uint32_t a) {
+    if constexpr (NG == 2) return lds64(a);
+    else return make_uint2(lds32(a), 0u);
+}
+
+__device__ __forceinline__ float fast_exp2(float x) {
+    float y;
+    asm("ex2.approx.ftz.f32 %0, %1;\n" : "=f"(y) : "f"(x));
+    return y;
+}
+
+__device__ __forceinline__ uint32_t movmatrix_t(uint32_t x) {
+    uint32_t y;
+    asm("movmatrix.sync.aligned.m8n8.trans.b16 %0, %1;\n" : "=r"(y) : "r"(x));
+    return y;
+}
+
+__device__ __forceinline__ float max_over_g(float v) {   // lanes with equal t (xor 4, 8, 16)
+    v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 4));
+    v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 8));
+    return fmaxf(v, __shfl_xor_sync(0xffffffffu, v, 16));
+}
+__device__ __forceinline__ float sum_over_g(float v) {
+    v += __shfl_xor_sync(0xffffffffu, v, 4);
+    v += __shfl_xor_sync(0xffffffffu, v, 8);
+    return v + __shfl_xor_sync(0xffffffffu, v, 16);
+}
+__device__ __forceinline__ float sum_over_t(float v) {
     v += __shfl_xor_sync(0xffffffffu, v, 1);
     return v + __shfl_xor_sync(0xffffffffu, v, 2);
 }
@@ -213,24 +333,51 @@ __device__ __forceinline__ void store_row8(const AttnArgs &a, int64_t row, int d
 }
 
 // -------------------------------------------------------------- the kernel
+// Per 16-token sub-block and lane (g = lane/4, t = lane%4):
+//  K-MMA   S^T[token][head] (16x8) = Kc[token][dims] (A, codes as fp16 subnormals)
+//                                   x q^T[dims][head] (B, fp16), one accumulator per group
+//  scores  z = sigma*log2e * sum_g ( 2^20 scale_tg S_g + min_tg Qs_g )    (folded dequant)
+//  softmax running max / sum per head (heads 2t, 2t+1 live in this lane)
+//  P^T     (p * scaleV) packed fp16, transposed in registers with movmatrix
+//  V-MMA   O^T[dim][head] (16x8 per 16 dims) += Vc^T[dims][token] (A) x P^T[token][head] (B)
+//  min     Pm[head][g] += sum_token p * minV
+// Stages (kSub sub-blocks) are software-pipelined: the K part of stage i+1 is
+// issued before the softmax/V part of stage i.  All control state (work map,
+// iterators, segment descriptors) lives in shared memory so that the
+// registers hold only the math state.
+
+struct SegDesc {      // the segment the consumer is processing
+    int b, kvh, blk0, nb, sn, v, x0, L;
+};
+
+struct WarpCtl {
+    SegIter pc;       // producer iterator (lane 0)
+    SegIter cc;       // consumer iterator (lane 0)
+    SegDesc seg;      // current consumer segment (all lanes read)
+    int ppos;         // blocks of pc's segment already issued
+    int qb, qkvh;     // pair whose q fragments are loaded
+};
+
 template <int D>
-__global__ void __launch_bounds__(kWarps * 32, 4) decode_attn_q4_kernel(const AttnArgs a) {
+struct KState {       // per-stage scores handed from the K part to the V part
+    float z[kSub][2][2];
+};
+
+template <int D>
+__global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q4_kernel(const AttnArgs a) {
     using GG = Geo<D>;
     constexpr int NG = GG::NG;
     extern __shared__ __align__(128) uint8_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);                 // [kWarps][kStages]
     uint8_t *ring = smem + 128;                                           // [kWarps][kStages][STAGE]
     int *prefix = reinterpret_cast<int *>(ring + kWarps * kStages * GG::STAGE);
+    __shared__ WorkMap wms;
+    __shared__ WarpCtl ctls[kWarps];
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int g = lane >> 2, t = lane & 3;
 
-    // ---- work map (every CTA computes the same one)
-    WorkMap wm;
-    wm.B = a.B;
-    wm.Hkv = a.Hkv;
-    wm.k = a.num_splits;
-    wm.W = gridDim.x * kWarps;
+    // ---- work map (identical in every CTA)
     if (a.lens) {
         if (warp == 0) {   // exclusive scan of Hkv*ceil(L_b/16) over b, lane-chunked
             const int per = (a.B + 31) / 32;
@@ -255,22 +402,34 @@ __global__ void __launch_bounds__(kWarps * 32, 4) decode_attn_q4_kernel(const At
             if (lane == 31) prefix[a.B] = incl;
         }
         __syncthreads();
-        wm.prefix = prefix;
-        wm.nbu = 0;
-        wm.N = prefix[a.B];
-    } else {
-        wm.prefix = nullptr;
-        wm.nbu = (a.len + kBlk - 1) / kBlk;
-        wm.N = (int64_t)a.B * a.Hkv * wm.nbu;
     }
-    if (wm.k == 0) wm.V = wm.N < wm.W ? wm.N : wm.W;
-    else wm.V = (int64_t)a.B * a.Hkv * wm.k;
+    if (threadIdx.x == 0) {
+        WorkMap wm;
+        wm.B = a.B;
+        wm.Hkv = a.Hkv;
+        wm.k = a.num_splits;
+        wm.W = gridDim.x * kWarps;
+        if (a.lens) {
+            wm.prefix = prefix;
+            wm.nbu = 0;
+            wm.N = prefix[a.B];
+        } else {
+            wm.prefix = nullptr;
+            wm.nbu = (a.len + kBlk - 1) / kBlk;
+            wm.N = a.B * a.Hkv * wm.nbu;
+        }
+        wm.V = wm.k == 0 ? (wm.N < wm.W ? wm.N : wm.W) : a.B * a.Hkv * wm.k;
+        wm.T = a.team;
+        wm.n_teams = a.team ? wm.W / a.team : 0;
+        wms = wm;
+    }
+    __syncthreads();
 
     const int gw = blockIdx.x * kWarps + warp;
 
     // ---- zero rows of empty sequences (per-sequence mode only)
     if (a.lens) {
-        for (int b = gw; b < a.B; b += wm.W) {
+        for (int b = gw; b < a.B; b += wms.W) {
             if (a.lens[b] > 0) continue;
             for (int i = lane; i < a.Hq * D; i += 32) {
                 const int64_t off = (int64_t)b * a.Hq * D + i;
@@ -282,163 +441,237 @@ __global__ void __launch_bounds__(kWarps * 32, 4) decode_attn_q4_kernel(const At
 
     uint64_t *wbar = bars + warp * kStages;
     uint8_t *wring = ring + warp * kStages * GG::STAGE;
-    if (lane == 0) {
-        for (int s = 0; s < kStages; ++s) mbar_init(&wbar[s], 1);
-        fence_mbar_init();
-    }
-    __syncwarp();
-
-    __shared__ Cursor pcs[kWarps];   // producer cursors (lane 0 only)
-    Cursor cc;
-    cc.enter(wm, gw);
-    if (cc.done) return;
-    Cursor &pc = pcs[warp];
-    if (lane == 0) pc = cc;
+    WarpCtl &ctl = ctls[warp];
     const uint64_t pol = policy_evict_first();
 
-    auto issue = [&](const Cursor &c, int slot) {
-        const int64_t tok0 = ((int64_t)c.b * a.Hkv + c.kvh) * a.cap + (int64_t)c.blk * kBlk;
-        uint8_t *dst = wring + slot * GG::STAGE;
-        mbar_arrive_expect_tx(&wbar[slot], GG::STAGE);
-        bulk_g2s(dst, a.kc + tok0 * (D / 2), GG::KC, &wbar[slot], pol);
-        bulk_g2s(dst + GG::KC, a.km + tok0 * NG, GG::KM, &wbar[slot], pol);
-        bulk_g2s(dst + GG::KC + GG::KM, a.vc + tok0 * (D / 2), GG::KC, &wbar[slot], pol);
-        bulk_g2s(dst + 2 * GG::KC + GG::KM, a.vm + tok0 * NG, GG::KM, &wbar[slot], pol);
+    // Producer (lane 0): one stage = up to kSub blocks of the producer's current
+    // segment; only the tokens < L_b are copied (exact-size tail, 16-B granular).
+    auto issue = [&](int slot) {
+        const WorkMap &wm = wms;
+        SegIter &pc = ctl.pc;
+        const int ppos = ctl.ppos;
+        const int n = min(kSub, pc.sn - ppos);
+        const int Lb = a.lens ? min(a.lens[pc.b], a.cap) : a.len;
+        const int tok_first = (pc.blk + ppos) * kBlk;
+        const int ntok = min(n * kBlk, Lb - tok_first);
+        const int bytes = (ntok * GG::ROW + 15) & ~15;          // cap % 16 == 0: in bounds
+        const int64_t tok0 = ((int64_t)pc.b * a.Hkv + pc.kvh) * a.cap + tok_first;
+        mbar_arrive_expect_tx(&wbar[slot], bytes);
+        bulk_g2s(wring + slot * GG::STAGE, a.kv + tok0 * GG::ROW, bytes, &wbar[slot], pol);
+        if (ppos + n >= pc.sn) {
+            do pc.next(wm); while (!pc.done && pc.sn == 0);
+            ctl.ppos = 0;
+        } else {
+            ctl.ppos = ppos + n;
+        }
     };
 
     if (lane == 0) {
-        for (int s = 0; s < kStages && !pc.done; ++s) {
-            issue(pc, s);
-            pc.advance(wm);
+        for (int s = 0; s < kStages; ++s) mbar_init(&wbar[s], 1);
+        fence_mbar_init();
+        if (wms.T) {
+            ctl.cc.v = gw / wms.T;           // team id = first pair
+            ctl.cc.x0 = gw % wms.T;          // rank in team
+        } else {
+            ctl.cc.v = gw;
         }
+        ctl.cc.begin_v(wms);
+        ctl.pc = ctl.cc;
+        ctl.ppos = 0;
+        ctl.qb = -1;
+        ctl.qkvh = -1;
+        while (!ctl.pc.done && ctl.pc.sn == 0) ctl.pc.next(wms);   // (team mode) empty segments
+        for (int s = 0; s < kStages && !ctl.pc.done; ++s) issue(s);
     }
     __syncwarp();
 
+    // ---- per-lane constant shared-memory offsets inside a stage (sub-block 0)
+    const int tk0 = tperm(g), tk1 = 8 + tperm(g);                    // this lane's K/meta tokens
+    const uint32_t ring_u32 = smem_u32(wring);
+    const uint32_t offK0 = ring_u32 + tk0 * GG::ROW + 8 * t;
+    const uint32_t offKm0 = ring_u32 + tk0 * GG::ROW + GG::OKM;
+    const uint32_t offVm0 = ring_u32 + tk0 * GG::ROW + GG::OVM;
+    const uint32_t offVa0 = ring_u32 + tperm(2 * t) * GG::ROW + GG::OVC + 4 * g;
+    const uint32_t offVb0 = ring_u32 + tperm(2 * t + 1) * GG::ROW + GG::OVC + 4 * g;
+    constexpr int dK1 = 8 * GG::ROW;   // token row +8
+    constexpr int dM1 = 8 * GG::ROW;
+    constexpr int dSC = kBlk * GG::ROW; // sub-block stride
+    constexpr int dSM = kBlk * GG::ROW;
+
     const float NEG_INF = -INFINITY;
-    const uint32_t ZERO = 0u;
-    uint32_t it = 0;            // blocks consumed by this warp
-    int qb = -1, qkvh = -1;     // pair whose q is loaded
-    uint32_t qa[NG][4][2];      // q A-fragments
-    float qs[NG];               // per-group sums of q (head g)
-    const bool head_ok = g < a.G;
+    const float zs = a.scale_log2;            // sigma * log2(e)
+    const float zs24 = zs * 16777216.0f;      // ... * 2^24 (K products are q c 2^-24)
+    int slot = 0;                             // consumer ring position
+    uint32_t phase = 0;
+#if LMO_ATTN_PROFILE
+    long long prof_wait = 0, prof_t0 = clock64(), prof_seg = 0, prof_st = 0;
+#endif
+    uint32_t qf[NG][4][2];                    // q B-fragments (head g)
+    float qs[NG][2];                          // per-group sums of q for heads 2t, 2t+1
+    int team_k = 0;                           // pairs finished (team mode: scratch double buffer)
 
-    while (!cc.done) {
+    while (!ctl.cc.done) {
         // ------------------------------------------------ segment start
-        const int b = cc.b, kvh = cc.kvh, blk0 = cc.blk, nb = cc.nb;
-        const int64_t vseg = cc.v;
-        const int64_t pstart = cc.x - blk0;
-        const int64_t seg_n = min((int64_t)(nb - blk0), cc.xend - cc.x);
-        const bool full = (blk0 == 0) && (seg_n == nb);
-        const int L = a.lens ? min(a.lens[b], a.cap) : a.len;
-
-        if (b != qb || kvh != qkvh) {
-            qb = b;
-            qkvh = kvh;
-#pragma unroll
-            for (int grp = 0; grp < NG; ++grp) {
-                uint4 q0 = make_uint4(0, 0, 0, 0), q1 = q0;
-                if (head_ok) {
-                    const __half *qp = a.q + (((int64_t)b * a.Hq + kvh * a.G + g) * D + grp * 64 + 16 * t);
-                    q0 = *reinterpret_cast<const uint4 *>(qp);
-                    q1 = *reinterpret_cast<const uint4 *>(qp + 8);
+        if (lane == 0) {
+            SegIter &cc = ctl.cc;
+            SegDesc d;
+            d.b = cc.b; d.kvh = cc.kvh; d.blk0 = cc.blk; d.nb = cc.nb; d.sn = cc.sn;
+            d.v = cc.v; d.x0 = cc.x0;
+            d.L = a.lens ? min(a.lens[cc.b], a.cap) : a.len;
+            ctl.seg = d;
+            cc.next(wms);
+        }
+        __syncwarp();
+        const int seg_n = ctl.seg.sn, blk0 = ctl.seg.blk0, L = ctl.seg.L;
+#if LMO_ATTN_PROFILE
+        ++prof_seg;
+#endif
+        {
+            const int b = ctl.seg.b, kvh = ctl.seg.kvh;
+            if (b != ctl.qb || kvh != ctl.qkvh) {
+                __syncwarp();
+                if (lane == 0) {
+                    ctl.qb = b;
+                    ctl.qkvh = kvh;
                 }
-                const __half *h0 = reinterpret_cast<const __half *>(&q0);
-                const __half *h1 = reinterpret_cast<const __half *>(&q1);
-                __half q16[16];
-                float sum = 0.f;
 #pragma unroll
-                for (int i = 0; i < 8; ++i) {
-                    q16[i] = h0[i];
-                    q16[8 + i] = h1[i];
-                    sum += __half2float(h0[i]) + __half2float(h1[i]);
-                }
-                qs[grp] = warp_sum4(sum);
+                for (int grp = 0; grp < NG; ++grp) {
+                    uint4 q0 = make_uint4(0, 0, 0, 0), q1 = q0;
+                    if (g < a.G) {
+                        const __half *qp = a.q + (((int64_t)b * a.Hq + kvh * a.G + g) * D + grp * 64 + 16 * t);
+                        q0 = *reinterpret_cast<const uint4 *>(qp);
+                        q1 = *reinterpret_cast<const uint4 *>(qp + 8);
+                    }
+                    const __half *h0 = reinterpret_cast<const __half *>(&q0);
+                    const __half *h1 = reinterpret_cast<const __half *>(&q1);
+                    __half q16[16];
+                    float sum = 0.f;
 #pragma unroll
-                for (int kbl = 0; kbl < 4; ++kbl) {
+                    for (int i = 0; i < 8; ++i) {
+                        q16[i] = h0[i];
+                        q16[8 + i] = h1[i];
+                        sum += __half2float(h0[i]) + __half2float(h1[i]);
+                    }
+                    sum = sum_over_t(sum);                              // Qs of head g
+                    qs[grp][0] = __shfl_sync(0xffffffffu, sum, 8 * t);      // head 2t   (g = 2t)
+                    qs[grp][1] = __shfl_sync(0xffffffffu, sum, 8 * t + 4);  // head 2t+1
 #pragma unroll
-                    for (int r = 0; r < 2; ++r) {
-                        const int idx = 2 * kbl + r;
-                        const int i0 = 8 * (idx >> 2) + (idx & 3);
-                        __half2 pr = __halves2half2(q16[i0], q16[i0 + 4]);
-                        qa[grp][kbl][r] = *reinterpret_cast<uint32_t *>(&pr);
+                    for (int kbl = 0; kbl < 4; ++kbl) {
+#pragma unroll
+                        for (int r = 0; r < 2; ++r) {
+                            const int idx = 2 * kbl + r;
+                            const int i0 = 8 * (idx >> 2) + (idx & 3);
+                            __half2 pr = __halves2half2(q16[i0], q16[i0 + 4]);
+                            if (r == 1) pr = __hmul2(pr, __float2half2_rn(0.0625f));  // meets c*2^-20
+                            qf[grp][kbl][r] = *reinterpret_cast<uint32_t *>(&pr);
+                        }
                     }
                 }
             }
         }
 
-        float m_run = head_ok ? NEG_INF : 0.f;
-        float l_run = 0.f;
-        float pm[NG];
+        // prefetch the next segment's q rows into L2 (its first use is latency-critical)
+        if (!ctl.cc.done && lane < a.G) {
+            const int nb_ = ctl.cc.b, nk_ = ctl.cc.kvh;
+            const char *qn = reinterpret_cast<const char *>(a.q + ((int64_t)nb_ * a.Hq + nk_ * a.G + lane) * D);
+#pragma unroll
+            for (int o = 0; o < D * 2; o += 128)
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(qn + o));
+        }
+
+        float m_run[2] = {NEG_INF, NEG_INF};
+        float l_run[2] = {0.f, 0.f};
+        float pm[2][NG];
         float acc[NG * 4][4];
 #pragma unroll
-        for (int grp = 0; grp < NG; ++grp) pm[grp] = 0.f;
+        for (int grp = 0; grp < NG; ++grp) pm[0][grp] = pm[1][grp] = 0.f;
 #pragma unroll
         for (int i = 0; i < NG * 4; ++i) acc[i][0] = acc[i][1] = acc[i][2] = acc[i][3] = 0.f;
 
-        for (int64_t jb = 0; jb < seg_n; ++jb) {
-            const int slot = it % kStages;
-            mbar_wait(&wbar[slot], (it / kStages) & 1);
-            const uint8_t *sKc = wring + slot * GG::STAGE;
-            const uint8_t *sKm = sKc + GG::KC;
-            const uint8_t *sVc = sKm + GG::KM;
-            const uint8_t *sVm = sVc + GG::KC;
-            const int tokbase = (blk0 + (int)jb) * kBlk;
-
-            // ---- scores: S[head g, group][token] via HMMA on exact codes
-            float sacc[2][4];
+        // K part of one stage (ring position sl/ph): wait for the data, scores
+        auto wait_stage = [&](int sl, uint32_t ph) {
+#if LMO_ATTN_PROFILE
+            const long long pw0 = clock64();
+#endif
+            mbar_wait(&wbar[sl], ph);
+#if LMO_ATTN_PROFILE
+            prof_wait += clock64() - pw0;
+#endif
+        };
+        // FULL: all kSub sub-blocks present and no ragged tail -> branch-free
+        auto stage_k = [&](auto full, int sl, int jb, KState<D> &ks) {
+            constexpr bool F = decltype(full)::value;
+            const uint32_t st = sl * GG::STAGE;
+            const int nsub = F ? kSub : min(kSub, seg_n - jb);
 #pragma unroll
-            for (int nbk = 0; nbk < 2; ++nbk) {
-                sacc[nbk][0] = sacc[nbk][1] = sacc[nbk][2] = sacc[nbk][3] = 0.f;
-                const int tok = 8 * nbk + tok_perm(g);
-#pragma unroll
-                for (int grp = 0; grp < NG; ++grp) {
-                    const uint2 w = *reinterpret_cast<const uint2 *>(sKc + tok * (D / 2) + grp * 32 + 8 * t);
-                    uint32_t u[8];
-                    unpack_k(w.x, *reinterpret_cast<uint32_t(*)[4]>(&u[0]));
-                    unpack_k(w.y, *reinterpret_cast<uint32_t(*)[4]>(&u[4]));
-#pragma unroll
-                    for (int kbl = 0; kbl < 4; ++kbl) {
-                        if (grp == 0)
-                            mma_16816(sacc[nbk], qa[0][kbl][0], ZERO, qa[0][kbl][1], ZERO, u[2 * kbl], u[2 * kbl + 1]);
-                        else
-                            mma_16816(sacc[nbk], ZERO, qa[grp][kbl][0], ZERO, qa[grp][kbl][1], u[2 * kbl], u[2 * kbl + 1]);
-                    }
-                }
-            }
-
-            // ---- K meta of this thread's 4 tokens, scores in log2 domain
-            float z[2][2];
-            bool ok[2][2];
-#pragma unroll
-            for (int nbk = 0; nbk < 2; ++nbk) {
-#pragma unroll
-                for (int e = 0; e < 2; ++e) {
-                    const int tok = 8 * nbk + tok_perm(2 * t + e);
-                    ok[nbk][e] = head_ok && (tokbase + tok < L);
-                    const uint32_t *mp = reinterpret_cast<const uint32_t *>(sKm) + tok * NG;
-                    float sc = 0.f;
+            for (int s = 0; s < kSub; ++s) {
+                if (s < nsub) {
+                    const uint32_t ss = st + s * dSC;
+                    float sacc[NG][4];
 #pragma unroll
                     for (int grp = 0; grp < NG; ++grp) {
-                        const float2 f = meta_f2(mp[grp]);       // (min, scale)
-                        sc = fmaf(sacc[nbk][e + 2 * grp], f.y, sc);
-                        sc = fmaf(f.x, qs[grp], sc);
+                        const uint2 w0 = lds64(ss + offK0 + grp * 32);
+                        const uint2 w1 = lds64(ss + offK0 + dK1 + grp * 32);
+                        uint32_t u0[8], u1[8];
+                        unpack_k(w0.x, u0);
+                        unpack_k(w0.y, u0 + 4);
+                        unpack_k(w1.x, u1);
+                        unpack_k(w1.y, u1 + 4);
+                        sacc[grp][0] = sacc[grp][1] = sacc[grp][2] = sacc[grp][3] = 0.f;
+#pragma unroll
+                        for (int kbl = 0; kbl < 4; ++kbl)
+                            mma_16816(sacc[grp], u0[2 * kbl], u1[2 * kbl], u0[2 * kbl + 1],
+                                      u1[2 * kbl + 1], qf[grp][kbl][0], qf[grp][kbl][1]);
                     }
-                    z[nbk][e] = ok[nbk][e] ? sc * a.scale_log2 : NEG_INF;
+                    const uint32_t sm = st + s * dSM + offKm0;
+#pragma unroll
+                    for (int r = 0; r < 2; ++r) {
+                        const uint2 km = load_meta<NG>(sm + r * dM1);
+                        float z0 = 0.f, z1 = 0.f;
+#pragma unroll
+                        for (int grp = 0; grp < NG; ++grp) {
+                            const float2 f = meta_f2(grp == 0 ? km.x : km.y);
+                            const float sk = f.y * zs24;
+                            const float mk = f.x * zs;
+                            z0 = fmaf(sacc[grp][2 * r + 0], sk, fmaf(mk, qs[grp][0], z0));
+                            z1 = fmaf(sacc[grp][2 * r + 1], sk, fmaf(mk, qs[grp][1], z1));
+                        }
+                        ks.z[s][r][0] = z0;
+                        ks.z[s][r][1] = z1;
+                    }
+                    const int tokbase = (blk0 + jb + s) * kBlk;
+                    if (!F && tokbase + kBlk > L) {                 // ragged tail
+                        if (tokbase + tk0 >= L) ks.z[s][0][0] = ks.z[s][0][1] = NEG_INF;
+                        if (tokbase + tk1 >= L) ks.z[s][1][0] = ks.z[s][1][1] = NEG_INF;
+                    }
+                } else {
+                    ks.z[s][0][0] = ks.z[s][0][1] = ks.z[s][1][0] = ks.z[s][1][1] = NEG_INF;
                 }
             }
+        };
 
-            // ---- online softmax (per head g; lanes 4g..4g+3 agree)
-            float mblk = fmaxf(fmaxf(z[0][0], z[0][1]), fmaxf(z[1][0], z[1][1]));
-            mblk = warp_max4(mblk);
-            const float m_new = fmaxf(m_run, mblk);
-            if (__any_sync(0xffffffffu, m_new > m_run)) {
-                const float alpha = (m_new > m_run) ? exp2f(m_run - m_new) : 1.f;
-                m_run = m_new;
-                l_run *= alpha;
+        // softmax + V part of one stage, then hand the slot back to the producer
+        auto stage_v = [&](auto full, int sl, int jb, const KState<D> &ks) {
+            constexpr bool F = decltype(full)::value;
+            const uint32_t st = sl * GG::STAGE;
+            const int nsub = F ? kSub : min(kSub, seg_n - jb);
+            const bool tail = !F && (blk0 + jb + kSub) * kBlk > L;
+            float mb0 = fmaxf(fmaxf(ks.z[0][0][0], ks.z[0][1][0]), fmaxf(ks.z[kSub - 1][0][0], ks.z[kSub - 1][1][0]));
+            float mb1 = fmaxf(fmaxf(ks.z[0][0][1], ks.z[0][1][1]), fmaxf(ks.z[kSub - 1][0][1], ks.z[kSub - 1][1][1]));
+            mb0 = max_over_g(mb0);
+            mb1 = max_over_g(mb1);
+            const float mn0 = fmaxf(m_run[0], mb0), mn1 = fmaxf(m_run[1], mb1);
+            if (__any_sync(0xffffffffu, (mn0 > m_run[0]) || (mn1 > m_run[1]))) {
+                const float a0 = fast_exp2(m_run[0] - mn0), a1 = fast_exp2(m_run[1] - mn1);
+                m_run[0] = mn0;
+                m_run[1] = mn1;
+                l_run[0] *= a0;
+                l_run[1] *= a1;
 #pragma unroll
-                for (int grp = 0; grp < NG; ++grp) pm[grp] *= alpha;
-                const float a0 = __shfl_sync(0xffffffffu, alpha, 8 * t);
-                const float a1 = __shfl_sync(0xffffffffu, alpha, 8 * t + 4);
+                for (int grp = 0; grp < NG; ++grp) {
+                    pm[0][grp] *= a0;
+                    pm[1][grp] *= a1;
+                }
 #pragma unroll
                 for (int i = 0; i < NG * 4; ++i) {
                     acc[i][0] *= a0;
@@ -447,140 +680,264 @@ __global__ void __launch_bounds__(kWarps * 32, 4) decode_attn_q4_kernel(const At
                     acc[i][3] *= a1;
                 }
             }
-            float p[2][2];
 #pragma unroll
-            for (int nbk = 0; nbk < 2; ++nbk)
+            for (int s = 0; s < kSub; ++s) {
+                if (s < nsub) {
+                    float p[2][2];
 #pragma unroll
-                for (int e = 0; e < 2; ++e) {
-                    p[nbk][e] = ok[nbk][e] ? exp2f(z[nbk][e] - m_run) : 0.f;
-                    l_run += p[nbk][e];
-                }
-
-            // ---- V: O^T[dim][head] += V^T codes . (p * scale)
-            const int tA0 = tok_perm(2 * t), tB0 = tok_perm(2 * t + 1);
-#pragma unroll
-            for (int grp = 0; grp < NG; ++grp) {
-                float2 vm[2][2];
-#pragma unroll
-                for (int nbk = 0; nbk < 2; ++nbk)
-#pragma unroll
-                    for (int e = 0; e < 2; ++e) {
-                        const int tok = 8 * nbk + tok_perm(2 * t + e);
-                        vm[nbk][e] = meta_f2(reinterpret_cast<const uint32_t *>(sVm)[tok * NG + grp]);
-                        if (!ok[nbk][e]) vm[nbk][e] = make_float2(0.f, 0.f);   // masked tail: meta may be garbage
-                        pm[grp] = fmaf(p[nbk][e], vm[nbk][e].x, pm[grp]);     // V min term sum_j p_j min_jg
+                    for (int r = 0; r < 2; ++r) {
+                        p[r][0] = fast_exp2(ks.z[s][r][0] - m_run[0]);
+                        p[r][1] = fast_exp2(ks.z[s][r][1] - m_run[1]);
                     }
-                const uint32_t bp0 = pack_half2(p[0][0] * vm[0][0].y, p[0][1] * vm[0][1].y);
-                const uint32_t bp1 = pack_half2(p[1][0] * vm[1][0].y, p[1][1] * vm[1][1].y);
-                const uint8_t *vbase = sVc + grp * 32 + 4 * g;
-                const uint32_t wa0 = *reinterpret_cast<const uint32_t *>(vbase + tA0 * (D / 2));
-                const uint32_t wb0 = *reinterpret_cast<const uint32_t *>(vbase + tB0 * (D / 2));
-                const uint32_t wa1 = *reinterpret_cast<const uint32_t *>(vbase + (8 + tA0) * (D / 2));
-                const uint32_t wb1 = *reinterpret_cast<const uint32_t *>(vbase + (8 + tB0) * (D / 2));
-                uint32_t j0[8], j1[8];
-                unpack_v(wa0, wb0, j0);
-                unpack_v(wa1, wb1, j1);
+                    l_run[0] += p[0][0] + p[1][0];
+                    l_run[1] += p[0][1] + p[1][1];
+                    const uint32_t ss = st + s * dSC;
+                    const uint32_t sm = st + s * dSM;
+                    const uint2 vmA = load_meta<NG>(sm + offVm0);
+                    const uint2 vmB = load_meta<NG>(sm + offVm0 + dM1);
 #pragma unroll
-                for (int mbl = 0; mbl < 4; ++mbl)
-                    mma_16816(acc[grp * 4 + mbl], j0[2 * mbl], j0[2 * mbl + 1], j1[2 * mbl], j1[2 * mbl + 1], bp0, bp1);
+                    for (int grp = 0; grp < NG; ++grp) {
+                        float2 f0 = meta_f2(grp == 0 ? vmA.x : vmA.y);
+                        float2 f1 = meta_f2(grp == 0 ? vmB.x : vmB.y);
+                        if (tail) {                    // masked tail tokens: meta may be stale
+                            if (ks.z[s][0][0] == NEG_INF) f0 = make_float2(0.f, 0.f);
+                            if (ks.z[s][1][0] == NEG_INF) f1 = make_float2(0.f, 0.f);
+                        }
+                        pm[0][grp] = fmaf(p[0][0], f0.x, fmaf(p[1][0], f1.x, pm[0][grp]));
+                        pm[1][grp] = fmaf(p[0][1], f0.x, fmaf(p[1][1], f1.x, pm[1][grp]));
+                        // P^T: (token row, heads 2t..2t+1) -> transpose -> (head g, tokens 2t..2t+1)
+                        const uint32_t bp0 = movmatrix_t(pack_half2(p[0][0] * f0.y, p[0][1] * f0.y));
+                        const uint32_t bp1 = movmatrix_t(pack_half2(p[1][0] * f1.y, p[1][1] * f1.y));
+                        const uint32_t wa0 = lds32(ss + offVa0 + grp * 32);
+                        const uint32_t wb0 = lds32(ss + offVb0 + grp * 32);
+                        const uint32_t wa1 = lds32(ss + offVa0 + dK1 + grp * 32);
+                        const uint32_t wb1 = lds32(ss + offVb0 + dK1 + grp * 32);
+                        uint32_t j0[8], j1[8];
+                        unpack_v(wa0, wb0, j0);
+                        unpack_v(wa1, wb1, j1);
+#pragma unroll
+                        for (int mbl = 0; mbl < 4; ++mbl)
+                            mma_16816(acc[grp * 4 + mbl], j0[2 * mbl], j0[2 * mbl + 1], j1[2 * mbl],
+                                      j1[2 * mbl + 1], bp0, bp1);
+                    }
+                }
             }
             __syncwarp();
-            if (lane == 0 && !pc.done) {
-                issue(pc, slot);
-                pc.advance(wm);
+            if (lane == 0 && !ctl.pc.done) issue(sl);
+#if LMO_ATTN_PROFILE
+            ++prof_st;
+#endif
+        };
+
+        auto advance = [&](int &sl, uint32_t &ph) {
+            if (++sl == kStages) {
+                sl = 0;
+                ph ^= 1u;
             }
-            ++it;
-            cc.advance(wm);
+        };
+
+        // software pipeline over the segment's stages: K part of stage i+1, then
+        // softmax/V part of stage i.  Stages with all sub-blocks present and no
+        // ragged tail take the branch-free FULL path (the hot loop); the rest
+        // (at most the last one or two of a segment) take the general path.
+        const int nst = (seg_n + kSub - 1) / kSub;
+        const int nfull = max(0, min(seg_n / kSub, (L / kBlk - blk0) / kSub));
+        const std::true_type FULL{};
+        const std::false_type GEN{};
+        KState<D> kC, kN;
+        if (nst > 0) {
+            wait_stage(slot, phase);
+            if (nfull > 0) stage_k(FULL, slot, 0, kC);
+            else stage_k(GEN, slot, 0, kC);
+        }
+        int i = 0;
+        // steady state: contiguous hot loop (FULL K part of i+1, FULL V part of i)
+#pragma unroll 1
+        for (; i + 1 < nfull; ++i) {
+            int slN = slot;
+            uint32_t phN = phase;
+            advance(slN, phN);
+            wait_stage(slN, phN);
+            stage_k(FULL, slN, (i + 1) * kSub, kN);
+            stage_v(FULL, slot, i * kSub, kC);
+            slot = slN;
+            phase = phN;
+            kC = kN;
+        }
+        // remainder: at most the last two stages of the segment
+#pragma unroll 1
+        for (; i < nst; ++i) {
+            int slN = slot;
+            uint32_t phN = phase;
+            advance(slN, phN);
+            if (i + 1 < nst) {
+                wait_stage(slN, phN);
+                stage_k(GEN, slN, (i + 1) * kSub, kN);
+            }
+            if (i < nfull) stage_v(FULL, slot, i * kSub, kC);
+            else stage_v(GEN, slot, i * kSub, kC);
+            slot = slN;
+            phase = phN;
+            kC = kN;
         }
 
         // ------------------------------------------------ segment end
-        const float l_tot = warp_sum4(l_run);
-        float pm_tot[NG];
+        // heads 2t+e: reduce l and Pm over the 8 g-lanes; O = 2^24 acc(row g) / 2^20 acc(row g+8) + Pm
+        float lt[2], pmt[2][NG];
 #pragma unroll
-        for (int grp = 0; grp < NG; ++grp) pm_tot[grp] = warp_sum4(pm[grp]);
-        const int hA = 2 * t, hB = 2 * t + 1;
-        const float lA = __shfl_sync(0xffffffffu, l_tot, 8 * t);
-        const float lB = __shfl_sync(0xffffffffu, l_tot, 8 * t + 4);
-        const float mA = __shfl_sync(0xffffffffu, m_run, 8 * t);
-        const float mB = __shfl_sync(0xffffffffu, m_run, 8 * t + 4);
-        float vA[NG][8], vB[NG][8];
+        for (int e = 0; e < 2; ++e) {
+            lt[e] = sum_over_g(l_run[e]);
 #pragma unroll
-        for (int grp = 0; grp < NG; ++grp) {
-            const float pA = __shfl_sync(0xffffffffu, pm_tot[grp], 8 * t);
-            const float pB = __shfl_sync(0xffffffffu, pm_tot[grp], 8 * t + 4);
-#pragma unroll
-            for (int mbl = 0; mbl < 4; ++mbl) {
-                vA[grp][2 * mbl] = acc[grp * 4 + mbl][0] + pA;
-                vA[grp][2 * mbl + 1] = acc[grp * 4 + mbl][2] + pA;
-                vB[grp][2 * mbl] = acc[grp * 4 + mbl][1] + pB;
-                vB[grp][2 * mbl + 1] = acc[grp * 4 + mbl][3] + pB;
-            }
+            for (int grp = 0; grp < NG; ++grp) pmt[e][grp] = sum_over_g(pm[e][grp]);
         }
-        const int64_t rowbase = (int64_t)b * a.Hq + (int64_t)kvh * a.G;
-        if (full) {
-            const float iA = 1.f / lA, iB = 1.f / lB;
+        float vo[2][NG][8];
 #pragma unroll
-            for (int grp = 0; grp < NG; ++grp) {
+        for (int grp = 0; grp < NG; ++grp)
 #pragma unroll
-                for (int i = 0; i < 8; ++i) {
-                    vA[grp][i] *= iA;
-                    vB[grp][i] *= iB;
+            for (int mbl = 0; mbl < 4; ++mbl)
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                    vo[e][grp][2 * mbl] = fmaf(acc[grp * 4 + mbl][e], 16777216.0f, pmt[e][grp]);
+                    vo[e][grp][2 * mbl + 1] = fmaf(acc[grp * 4 + mbl][2 + e], 1048576.0f, pmt[e][grp]);
                 }
-                if (hA < a.G) store_row8<D>(a, rowbase + hA, grp * 64 + 8 * g, vA[grp]);
-                if (hB < a.G) store_row8<D>(a, rowbase + hB, grp * 64 + 8 * g, vB[grp]);
+        const SegDesc sd = ctl.seg;
+        const int64_t rowbase = (int64_t)sd.b * a.Hq + (int64_t)sd.kvh * a.G;
+        const bool full = (sd.blk0 == 0) && (sd.sn == sd.nb) && wms.T <= 1;
+        if (wms.T > 1) {
+            // ---- pair team: partials through L2 scratch, named barrier, rank 0 merges
+            const int T = wms.T;
+            const int64_t myslot = 2 * (int64_t)gw + (team_k & 1);
+            float *rec = a.partials + myslot * (int64_t)a.G * GG::REC;
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+                const int h = 2 * t + e;
+                if (h < a.G) {
+#pragma unroll
+                    for (int grp = 0; grp < NG; ++grp) {
+                        float4 *r4 = reinterpret_cast<float4 *>(rec + h * GG::REC + grp * 64 + 8 * g);
+                        __stcg(r4, make_float4(vo[e][grp][0], vo[e][grp][1], vo[e][grp][2], vo[e][grp][3]));
+                        __stcg(r4 + 1, make_float4(vo[e][grp][4], vo[e][grp][5], vo[e][grp][6], vo[e][grp][7]));
+                    }
+                    if (g == 0) {
+                        __stcg(rec + h * GG::REC + D, m_run[e]);
+                        __stcg(rec + h * GG::REC + D + 1, lt[e]);
+                    }
+                }
+            }
+            asm volatile("bar.sync %0, %1;\n" ::"r"(1 + warp / T), "r"(T * 32) : "memory");
+            if (gw % T == 0) {
+                constexpr int DPL = D / 32;
+                for (int h = 0; h < a.G; ++h) {
+                    float M = NEG_INF;
+                    for (int j = 0; j < T; ++j)
+                        M = fmaxf(M, __ldcg(a.partials + (2 * (int64_t)(gw + j) + (team_k & 1)) * a.G * GG::REC + h * GG::REC + D));
+                    if (M == NEG_INF) continue;          // empty sequence: zero row already written
+                    float l = 0.f, o[DPL];
+#pragma unroll
+                    for (int i2 = 0; i2 < DPL; ++i2) o[i2] = 0.f;
+                    for (int j = 0; j < T; ++j) {
+                        const float *r = a.partials + (2 * (int64_t)(gw + j) + (team_k & 1)) * a.G * GG::REC + h * GG::REC;
+                        const float w = exp2f(__ldcg(r + D) - M);
+                        l = fmaf(__ldcg(r + D + 1), w, l);
+#pragma unroll
+                        for (int i2 = 0; i2 < DPL; ++i2) o[i2] = fmaf(__ldcg(r + lane * DPL + i2), w, o[i2]);
+                    }
+                    const float il = 1.f / l;
+                    const int64_t row = rowbase + h;
+#pragma unroll
+                    for (int i2 = 0; i2 < DPL; ++i2) {
+                        const int64_t off = row * D + lane * DPL + i2;
+                        if (a.out_f16) static_cast<__half *>(a.out)[off] = __float2half_rn(o[i2] * il);
+                        else static_cast<float *>(a.out)[off] = o[i2] * il;
+                    }
+                }
+            }
+            ++team_k;
+        } else if (full) {
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+                const int h = 2 * t + e;
+                const float il = 1.f / lt[e];
+#pragma unroll
+                for (int grp = 0; grp < NG; ++grp) {
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) vo[e][grp][i] *= il;
+                    if (h < a.G) store_row8<D>(a, rowbase + h, grp * 64 + 8 * g, vo[e][grp]);
+                }
             }
         } else {
-            // partial record for this (virtual warp, pair) slot
-            const int64_t slot = wm.slot_of(vseg, pstart);
-            float *rec = a.partials + slot * (int64_t)a.G * GG::REC;
+            const WorkMap wm = wms;
+            // pair start = global index of the pair's first block
+            const int ps = wm.seq_start(sd.b) + sd.kvh * sd.nb;
+            // partial record in slot (virtual warp, first/last) -- stream-K -- or (virtual warp)
+            const int64_t rslot = wm.k == 0 ? 2 * (int64_t)sd.v + (sd.x0 < ps ? 1 : 0) : sd.v;
+            float *rec = a.partials + rslot * (int64_t)a.G * GG::REC;
 #pragma unroll
-            for (int grp = 0; grp < NG; ++grp) {
-                if (hA < a.G) {
-                    float *r = rec + hA * GG::REC + grp * 64 + 8 * g;
-                    __stcg(reinterpret_cast<float4 *>(r), make_float4(vA[grp][0], vA[grp][1], vA[grp][2], vA[grp][3]));
-                    __stcg(reinterpret_cast<float4 *>(r) + 1, make_float4(vA[grp][4], vA[grp][5], vA[grp][6], vA[grp][7]));
+            for (int e = 0; e < 2; ++e) {
+                const int h = 2 * t + e;
+                if (h < a.G) {
+#pragma unroll
+                    for (int grp = 0; grp < NG; ++grp) {
+                        float4 *r4 = reinterpret_cast<float4 *>(rec + h * GG::REC + grp * 64 + 8 * g);
+                        __stcg(r4, make_float4(vo[e][grp][0], vo[e][grp][1], vo[e][grp][2], vo[e][grp][3]));
+                        __stcg(r4 + 1, make_float4(vo[e][grp][4], vo[e][grp][5], vo[e][grp][6], vo[e][grp][7]));
+                    }
+                    if (g == 0) {
+                        __stcg(rec + h * GG::REC + D, m_run[e]);
+                        __stcg(rec + h * GG::REC + D + 1, lt[e]);
+                    }
                 }
-                if (hB < a.G) {
-                    float *r = rec + hB * GG::REC + grp * 64 + 8 * g;
-                    __stcg(reinterpret_cast<float4 *>(r), make_float4(vB[grp][0], vB[grp][1], vB[grp][2], vB[grp][3]));
-                    __stcg(reinterpret_cast<float4 *>(r) + 1, make_float4(vB[grp][4], vB[grp][5], vB[grp][6], vB[grp][7]));
-                }
-            }
-            if (g == 0) {
-                if (hA < a.G) { __stcg(rec + hA * GG::REC + D, mA); __stcg(rec + hA * GG::REC + D + 1, lA); }
-                if (hB < a.G) { __stcg(rec + hB * GG::REC + D, mB); __stcg(rec + hB * GG::REC + D + 1, lB); }
             }
             __threadfence();
             __syncwarp();
-            // number of segments of this pair
-            const int64_t pend = pstart + nb;
-            const int64_t v0 = wm.vwarp_of(pstart), v1 = wm.vwarp_of(pend - 1);
-            int nseg = 0;
-            for (int64_t v = v0; v <= v1; ++v) nseg += (wm.R(v) < wm.R(v + 1)) ? 1 : 0;
-            const int pair = b * a.Hkv + kvh;
+            // segments of this pair = non-empty ranges of virtual warps v0..v1
+            const int v0 = wm.vwarp_of(ps), v1 = wm.vwarp_of(ps + sd.nb - 1);
+            int nseg = v1 - v0 + 1;
+            if (wm.k != 0) {
+                nseg = 0;
+                for (int v = v0; v <= v1; ++v) nseg += (wm.R(v) < wm.R(v + 1)) ? 1 : 0;
+            }
+            const int pair = sd.b * a.Hkv + sd.kvh;
             int last = 0;
             if (lane == 0) last = (atomicAdd(&a.counters[pair], 1) == nseg - 1);
             last = __shfl_sync(0xffffffffu, last, 0);
             if (last) {
                 __threadfence();
+                // slot of the j-th segment; stream-K: only v0's range can start before the pair
+                const int64_t s0 = wm.k == 0 ? 2 * (int64_t)v0 + (wm.R(v0) < ps ? 1 : 0) : v0;
                 constexpr int DPL = D / 32;      // dims per lane
                 for (int h = 0; h < a.G; ++h) {
+                    // pass 1 (lanes over segments): max of the partial maxima
                     float M = NEG_INF;
-                    for (int64_t v = v0; v <= v1; ++v) {
-                        if (!(wm.R(v) < wm.R(v + 1))) continue;
-                        const float *r = a.partials + wm.slot_of(v, pstart) * (int64_t)a.G * GG::REC + h * GG::REC;
-                        M = fmaxf(M, __ldcg(r + D));
+                    for (int j = lane; j < v1 - v0 + 1; j += 32) {
+                        const int v = v0 + j;
+                        if (wm.k != 0 && !(wm.R(v) < wm.R(v + 1))) continue;
+                        const int64_t sl = wm.k == 0 ? (j == 0 ? s0 : 2 * (int64_t)v) : v;
+                        M = fmaxf(M, __ldcg(a.partials + sl * a.G * GG::REC + h * GG::REC + D));
                     }
+#pragma unroll
+                    for (int off = 16; off > 0; off >>= 1) M = fmaxf(M, __shfl_xor_sync(0xffffffffu, M, off));
                     float l = 0.f, o[DPL];
 #pragma unroll
                     for (int i = 0; i < DPL; ++i) o[i] = 0.f;
-                    for (int64_t v = v0; v <= v1; ++v) {
-                        if (!(wm.R(v) < wm.R(v + 1))) continue;
-                        const float *r = a.partials + wm.slot_of(v, pstart) * (int64_t)a.G * GG::REC + h * GG::REC;
+                    // pass 2 (all lanes, each its own dims): weighted sums
+                    for (int j = 0; j < v1 - v0 + 1; ++j) {
+                        const int v = v0 + j;
+                        if (wm.k != 0 && !(wm.R(v) < wm.R(v + 1))) continue;
+                        const int64_t sl = wm.k == 0 ? (j == 0 ? s0 : 2 * (int64_t)v) : v;
+                        const float *r = a.partials + sl * a.G * GG::REC + h * GG::REC;
                         const float w = exp2f(__ldcg(r + D) - M);
                         l = fmaf(__ldcg(r + D + 1), w, l);
+                        if (DPL == 4) {
+                            const float4 x = __ldcg(reinterpret_cast<const float4 *>(r) + lane);
+                            o[0] = fmaf(x.x, w, o[0]);
+                            o[1] = fmaf(x.y, w, o[1]);
+                            o[2] = fmaf(x.z, w, o[2]);
+                            o[3] = fmaf(x.w, w, o[3]);
+                        } else {
 #pragma unroll
-                        for (int i = 0; i < DPL; ++i) o[i] = fmaf(__ldcg(r + lane * DPL + i), w, o[i]);
+                            for (int i = 0; i < DPL; ++i) o[i] = fmaf(__ldcg(r + lane * DPL + i), w, o[i]);
+                        }
                     }
                     const float il = 1.f / l;
                     const int64_t row = rowbase + h;
@@ -594,52 +951,88 @@ __global__ void __launch_bounds__(kWarps * 32, 4) decode_attn_q4_kernel(const At
                 if (lane == 0) a.counters[pair] = 0;
             }
         }
+        __syncwarp();
     }
+#if LMO_ATTN_PROFILE
+    if (lane == 0 && g_attn_prof) {
+        unsigned long long *pr = g_attn_prof + 4 * (size_t)gw;
+        pr[0] = prof_wait;
+        pr[1] = clock64() - prof_t0;
+        pr[2] = prof_st;
+        pr[3] = prof_seg;
+    }
+#endif
 }
+
+#if LMO_ATTN_PROFILE
+extern "C" int lmo_debug_attn_profile(void *buf) {
+    return (int)cudaMemcpyToSymbol(g_attn_prof, &buf, sizeof(void *));
+}
+#endif
 
 // ---------------------------------------------------------------- host side
 template <int D>
-static size_t smem_bytes() {
-    return 128 + (size_t)kWarps * kStages * Geo<D>::STAGE + (kMaxBatchSmem + 1) * sizeof(int);
+static size_t smem_bytes(int B_prefix) {
+    return 128 + (size_t)kWarps * kStages * Geo<D>::STAGE + (B_prefix > 0 ? (B_prefix + 1) * sizeof(int) : 0);
 }
 
 template <int D>
-static int ctas_per_sm() {
-    static int occ[64] = {0};
+static int ctas_per_sm(int B_prefix) {
+    static int occ[64][2] = {{0}};
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev < 0 || dev >= 64) dev = 0;
-    if (occ[dev] == 0) {
+    const int mode = B_prefix > 0 ? 1 : 0;
+    if (occ[dev][mode] == 0) {
         cudaFuncSetAttribute(decode_attn_q4_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)smem_bytes<D>());
+                             (int)smem_bytes<D>(kMaxBatchSmem));
         int n = 0;
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, decode_attn_q4_kernel<D>, kWarps * 32,
-                                                      smem_bytes<D>());
-        occ[dev] = n > 0 ? n : 1;
+                                                      smem_bytes<D>(mode ? kMaxBatchSmem : 0));
+        occ[dev][mode] = n > 0 ? n : 1;
     }
-    return occ[dev];
+    return occ[dev][mode];
 }
 
-int attn_max_warps(int head_dim) {
-    const int occ = head_dim == 64 ? ctas_per_sm<64>() : ctas_per_sm<128>();
+int attn_max_warps(int head_dim, int B_prefix) {
+    const int occ = head_dim == 64 ? ctas_per_sm<64>(B_prefix) : ctas_per_sm<128>(B_prefix);
     return device_sm_count() * occ * kWarps;
 }
 
 size_t attn_workspace_bytes(int B, int Hkv, int Hq, int D, int num_splits) {
     const int G = Hq / Hkv;
     const size_t counters = ((size_t)B * Hkv * sizeof(int) + 255) / 256 * 256;
-    const size_t slots = num_splits > 0 ? (size_t)B * Hkv * num_splits : 2 * (size_t)attn_max_warps(D);
+    size_t slots = 2 * (size_t)attn_max_warps(D, 0);               // stream-K and team scratch
+    if (num_splits > 0 && (size_t)B * Hkv * num_splits > slots) slots = (size_t)B * Hkv * num_splits;
     return counters + slots * G * (D + 4) * sizeof(float);
+}
+
+// Work distribution (uniform length): pair teams of T in {1, 2, 4} warps, or
+// stream-K when there are too few pairs to fill the resident warps.  Cost in
+// units of one stage (32 tokens) of one warp, with a per-pair overhead.
+static int choose_team(int64_t pairs, int64_t nb, int64_t warps) {
+    const int64_t S = (nb + kSub - 1) / kSub;
+    double best = 1e30;
+    int bestT = 0;
+    for (int T = 1; T <= kWarps; T *= 2) {
+        const int64_t teams = warps / T;
+        const int64_t rounds = (pairs + teams - 1) / teams;
+        const double per = (double)((((nb + T - 1) / T) + kSub - 1) / kSub) + (T == 1 ? 1.0 : 2.0);
+        const double cost = rounds * per;
+        if (cost < best) {
+            best = cost;
+            bestT = T;
+        }
+    }
+    const double sk = (double)pairs * S / (double)warps + 4.0;   // stream-K: balanced + merge overhead
+    return sk < 0.9 * best ? 0 : bestT;
 }
 
 cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq, int len,
                                     const int32_t *lens, float softmax_scale, int num_splits,
                                     void *out, int out_f16, void *ws, cudaStream_t st) {
     AttnArgs a;
-    a.kc = c.k_codes;
-    a.vc = c.v_codes;
-    a.km = reinterpret_cast<const uint32_t *>(c.k_meta);
-    a.vm = reinterpret_cast<const uint32_t *>(c.v_meta);
+    a.kv = c.kv;
     a.B = c.batch;
     a.Hkv = c.kv_heads;
     a.cap = c.capacity;
@@ -657,22 +1050,33 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     a.partials = reinterpret_cast<float *>(static_cast<uint8_t *>(ws) + counters);
 
     const int D = c.head_dim;
-    const int max_ctas = attn_max_warps(D) / kWarps;
+    const int Bp = lens ? c.batch : 0;
+    const int max_ctas = attn_max_warps(D, Bp) / kWarps;
+    const int64_t pairs = (int64_t)c.batch * c.kv_heads;
+    const int64_t nbu = lens ? 0 : (len + kBlk - 1) / kBlk;
+    a.team = 0;
+    if (num_splits == 1 || num_splits == 2 || num_splits == 4) {
+        a.team = num_splits;                  // explicit team size (batch-independent results)
+        a.num_splits = 0;
+    } else if (num_splits == 0 && !lens) {
+        a.team = choose_team(pairs, nbu, (int64_t)max_ctas * kWarps);
+    }
     int64_t want_warps;
-    if (lens) {
+    if (a.team) {
+        want_warps = pairs * a.team;
+    } else if (lens) {
         want_warps = (int64_t)max_ctas * kWarps;
     } else {
-        const int64_t nbu = (len + kBlk - 1) / kBlk;
-        const int64_t N = (int64_t)c.batch * c.kv_heads * nbu;
-        want_warps = num_splits > 0 ? (int64_t)c.batch * c.kv_heads * num_splits : N;
+        const int64_t N = pairs * nbu;
+        want_warps = num_splits > 0 ? pairs * num_splits : N;
     }
     int64_t ctas = (want_warps + kWarps - 1) / kWarps;
     if (ctas > max_ctas) ctas = max_ctas;
     if (ctas < 1) ctas = 1;
     if (D == 64)
-        decode_attn_q4_kernel<64><<<(unsigned)ctas, kWarps * 32, smem_bytes<64>(), st>>>(a);
+        decode_attn_q4_kernel<64><<<(unsigned)ctas, kWarps * 32, smem_bytes<64>(Bp), st>>>(a);
     else
-        decode_attn_q4_kernel<128><<<(unsigned)ctas, kWarps * 32, smem_bytes<128>(), st>>>(a);
+        decode_attn_q4_kernel<128><<<(unsigned)ctas, kWarps * 32, smem_bytes<128>(Bp), st>>>(a);
     note_launch();
     return cudaGetLastError();
 }

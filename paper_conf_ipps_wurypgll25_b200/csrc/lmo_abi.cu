@@ -40,13 +40,11 @@ size_t attn_workspace_bytes(int B, int Hkv, int Hq, int D, int num_splits);
 static bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 static lmo_status check_cache(const lmo_kv_cache *c) {
-    if (!c || !c->k_codes || !c->v_codes || !c->k_meta || !c->v_meta) return LMO_ERR_NULL;
+    if (!c || !c->kv) return LMO_ERR_NULL;
     if (c->batch <= 0 || c->kv_heads <= 0 || c->capacity <= 0) return LMO_ERR_SHAPE;
     if (c->head_dim != 64 && c->head_dim != 128) return LMO_ERR_UNSUPPORTED;
     if (c->capacity % 16 != 0) return LMO_ERR_SHAPE;
-    if (!aligned16(c->k_codes) || !aligned16(c->v_codes) || !aligned16(c->k_meta) ||
-        !aligned16(c->v_meta))
-        return LMO_ERR_ALIGN;
+    if (!aligned16(c->kv)) return LMO_ERR_ALIGN;
     return LMO_OK;
 }
 
@@ -151,6 +149,11 @@ lmo_status lmo_gen_fill_f16(void *dst, int32_t nb, int32_t nh, int32_t npos, int
         return LMO_ERR_SHAPE;
     return cuda_status(launch_gen_fill(dst, nb, nh, npos, dim, seed, stream_id, layer, b0, h0, p0,
                                        group, static_cast<cudaStream_t>(stream)));
+}
+
+size_t lmo_kv_row_bytes(int32_t head_dim) {
+    if (head_dim != 64 && head_dim != 128) return 0;
+    return (size_t)2 * (head_dim / 2 + 4 * (head_dim / kGroup));
 }
 
 uint64_t lmo_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }

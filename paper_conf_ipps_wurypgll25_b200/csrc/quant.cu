@@ -100,12 +100,12 @@ __global__ void __launch_bounds__(256) kv_append_kernel(lmo_kv_cache cache,
     uint32_t mw;
     const uint32_t w = quantize_group_lane8(xv, mw);
     if (valid) {
+        // compressed row: K codes | K meta | V codes | V meta
+        const int RB = d / 2, MB = gpr * 4, ROW = 2 * (RB + MB);
         const int64_t slot = bh * cache.capacity + pos + t;
-        uint8_t *cdst = (kv == 0 ? cache.k_codes : cache.v_codes) + slot * (d / 2) + grp * 32;
-        uint32_t *mdst = reinterpret_cast<uint32_t *>(kv == 0 ? cache.k_meta : cache.v_meta) +
-                         slot * gpr + grp;
-        reinterpret_cast<uint32_t *>(cdst)[lane8] = w;
-        if (lane8 == 0) *mdst = mw;
+        uint8_t *row = cache.kv + slot * ROW + kv * (RB + MB);
+        reinterpret_cast<uint32_t *>(row + grp * 32)[lane8] = w;
+        if (lane8 == 0) reinterpret_cast<uint32_t *>(row + RB)[grp] = mw;
     }
 }
 

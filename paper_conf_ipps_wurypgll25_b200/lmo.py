@@ -29,9 +29,7 @@ class LmoError(RuntimeError):
 
 
 class lmo_kv_cache(ctypes.Structure):
-    _fields_ = [("k_codes", ctypes.c_void_p), ("v_codes", ctypes.c_void_p),
-                ("k_meta", ctypes.c_void_p), ("v_meta", ctypes.c_void_p),
-                ("batch", ctypes.c_int32), ("kv_heads", ctypes.c_int32),
+    _fields_ = [("kv", ctypes.c_void_p), ("batch", ctypes.c_int32), ("kv_heads", ctypes.c_int32),
                 ("capacity", ctypes.c_int32), ("head_dim", ctypes.c_int32)]
 
 
@@ -57,6 +55,8 @@ def _load():
     L.lmo_decode_attention_workspace_bytes.restype = ctypes.c_size_t
     L.lmo_status_string.argtypes = [ctypes.c_int]
     L.lmo_status_string.restype = ctypes.c_char_p
+    L.lmo_kv_row_bytes.argtypes = [i32]
+    L.lmo_kv_row_bytes.restype = ctypes.c_size_t
     L.lmo_launch_count.argtypes = []
     L.lmo_launch_count.restype = ctypes.c_uint64
     L.lmo_version.argtypes = []
@@ -67,6 +67,7 @@ def _load():
 _lib = _load()
 LIB_PATH = _build.LIB
 EXPORTS = ["lmo_quantize_groupwise", "lmo_dequantize_groupwise", "lmo_kv_append_quant",
+           "lmo_kv_row_bytes",
            "lmo_decode_attention_workspace_bytes", "lmo_decode_attention_q4", "lmo_status_string",
            "lmo_gen_fill_f16", "lmo_launch_count", "lmo_version"]
 
@@ -129,13 +130,16 @@ def lmo_dequantize_groupwise(codes: torch.Tensor, meta: torch.Tensor, outer: int
 
 # ------------------------------------------------------------ KV cache ----
 
+def row_bytes(head_dim: int) -> int:
+    """Compressed K+V token row: K codes | K meta | V codes | V meta."""
+    return 2 * (head_dim // 2 + 4 * (head_dim // GROUP))
+
+
 @dataclass
 class KVCache:
-    """One layer's q4 KV cache in the library layout (torch owns the memory)."""
-    k_codes: torch.Tensor   # [B][Hkv][cap][d/2] uint8
-    v_codes: torch.Tensor
-    k_meta: torch.Tensor    # [B][Hkv][cap][d/64] int32 (lmo_qmeta)
-    v_meta: torch.Tensor
+    """One layer's q4 KV cache in the library layout (torch owns the memory):
+    kv [B][Hkv][cap][row_bytes] uint8, one compressed K+V row per token slot."""
+    kv: torch.Tensor
     batch: int
     kv_heads: int
     capacity: int
@@ -146,21 +150,38 @@ class KVCache:
               zero: bool = False) -> "KVCache":
         cap = (capacity + 15) // 16 * 16
         alloc = torch.zeros if zero else torch.empty
-        ng = head_dim // GROUP
-        kc = alloc((batch, kv_heads, cap, head_dim // 2), dtype=torch.uint8, device=device)
-        vc = alloc((batch, kv_heads, cap, head_dim // 2), dtype=torch.uint8, device=device)
-        km = alloc((batch, kv_heads, cap, ng), dtype=torch.int32, device=device)
-        vm = alloc((batch, kv_heads, cap, ng), dtype=torch.int32, device=device)
-        return KVCache(kc, vc, km, vm, batch, kv_heads, cap, head_dim)
+        kv = alloc((batch, kv_heads, cap, row_bytes(head_dim)), dtype=torch.uint8, device=device)
+        return KVCache(kv, batch, kv_heads, cap, head_dim)
 
     def abi(self) -> lmo_kv_cache:
-        return lmo_kv_cache(self.k_codes.data_ptr(), self.v_codes.data_ptr(),
-                            self.k_meta.data_ptr(), self.v_meta.data_ptr(), self.batch,
-                            self.kv_heads, self.capacity, self.head_dim)
+        return lmo_kv_cache(self.kv.data_ptr(), self.batch, self.kv_heads, self.capacity,
+                            self.head_dim)
 
     def nbytes(self) -> int:
-        return sum(t.numel() * t.element_size()
-                   for t in (self.k_codes, self.v_codes, self.k_meta, self.v_meta))
+        return self.kv.numel()
+
+    # field views (strided): codes [B][Hkv][cap][d/2] u8, meta [B][Hkv][cap][d/64] as int32 bytes
+    def field(self, name: str) -> torch.Tensor:
+        rb, mb = self.head_dim // 2, 4 * (self.head_dim // GROUP)
+        off = {"k_codes": (0, rb), "k_meta": (rb, mb), "v_codes": (rb + mb, rb),
+               "v_meta": (2 * rb + mb, mb)}[name]
+        return self.kv[..., off[0]:off[0] + off[1]]
+
+    def to_host_fields(self):
+        """Copy to host as the oracle's field arrays: codes uint8 [B][Hkv][cap][d/2],
+        meta uint16 [B][Hkv][cap][d/64][2] ({min, scale} bit patterns)."""
+        import numpy as np
+        kv = self.kv.cpu().numpy()
+        rb, ng = self.head_dim // 2, self.head_dim // GROUP
+        out = {}
+        for name in ("k_codes", "k_meta", "v_codes", "v_meta"):
+            off = {"k_codes": 0, "k_meta": rb, "v_codes": rb + 4 * ng, "v_meta": 2 * rb + 4 * ng}[name]
+            if name.endswith("codes"):
+                out[name] = np.ascontiguousarray(kv[..., off:off + rb])
+            else:
+                m = np.ascontiguousarray(kv[..., off:off + 4 * ng])
+                out[name] = m.view(np.uint16).reshape(*m.shape[:-1], ng, 2)
+        return out
 
 
 def lmo_kv_append_quant(cache: KVCache, k_new: torch.Tensor, v_new: torch.Tensor, pos0: int = 0,

@@ -27,10 +27,9 @@ for key in ("c2", "c5", "c3", "c4"):
     L = w.max_len
     for l in range(nl):
         c = lmo.KVCache.empty(w.batch, w.kv_heads, w.capacity, w.head_dim)
-        for t in (c.k_codes, c.v_codes):
-            t.random_(0, 256)
-        for t in (c.k_meta, c.v_meta):
-            t.copy_(torch.tensor(0x2C00BC00, dtype=torch.int32))  # min -1.0, scale 1/16
+        c.kv.random_(0, 256)
+        for nm in ("k_meta", "v_meta"):
+            c.field(nm).view(torch.int32).fill_(0x2C00BC00)
         caches.append(c)
     q = torch.randn(w.batch, w.q_heads, w.head_dim, device='cuda').half()
     out = torch.empty(w.batch, w.q_heads, w.head_dim, device='cuda')

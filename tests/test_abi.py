@@ -56,7 +56,7 @@ def test_argument_validation_without_gpu(lib):
     assert L.lmo_quantize_groupwise(P(18), 1, 64, 1, 4, 64, P(16), P(16), None) == 4
     assert L.lmo_quantize_groupwise(None, 0, 64, 1, 4, 64, None, None, None) == 0   # empty no-op
     assert L.lmo_dequantize_groupwise(P(16), P(16), 1, 64, 1, 4, 64, None, None) == 1
-    c = lib.lmo_kv_cache(16, 32, 48, 64, 2, 2, 32, 128)
+    c = lib.lmo_kv_cache(16, 2, 2, 32, 128)
     assert L.lmo_kv_append_quant(ctypes.byref(c), P(16), P(16), 1, 32, None, None) == 2  # pos overflow
     c.head_dim = 96
     assert L.lmo_kv_append_quant(ctypes.byref(c), P(16), P(16), 1, 0, None, None) == 3
@@ -64,9 +64,11 @@ def test_argument_validation_without_gpu(lib):
     c.capacity = 30
     assert L.lmo_kv_append_quant(ctypes.byref(c), P(16), P(16), 1, 0, None, None) == 2
     c.capacity = 32
-    c.k_meta = 50
+    c.kv = 50
     assert L.lmo_kv_append_quant(ctypes.byref(c), P(16), P(16), 1, 0, None, None) == 4
-    c.k_meta = 48
+    c.kv = 48
+    assert L.lmo_kv_row_bytes(128) == 144 and L.lmo_kv_row_bytes(64) == 72
+    assert L.lmo_kv_row_bytes(96) == 0
     # attention: group ratio > 8 unsupported, len > capacity
     assert L.lmo_decode_attention_q4(ctypes.byref(c), P(16), 18, 4, None, 1.0, 0, P(16), 1,
                                      P(16), 1 << 30, None) == 3

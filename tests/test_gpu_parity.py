@@ -110,11 +110,7 @@ def test_weight_dequant_round_trip_shape(lmo):
 # ---------------------------------------------------------------- K2 -------
 
 def cache_to_host(cache):
-    return {
-        "k_codes": cache.k_codes.cpu().numpy(), "v_codes": cache.v_codes.cpu().numpy(),
-        "k_meta": cache.k_meta.cpu().numpy().view(np.uint16).reshape(*cache.k_meta.shape, 2),
-        "v_meta": cache.v_meta.cpu().numpy().view(np.uint16).reshape(*cache.v_meta.shape, 2),
-    }
+    return cache.to_host_fields()
 
 
 @pytest.mark.parametrize("d", [64, 128])
@@ -122,8 +118,7 @@ def test_append_bit_exact_with_canaries(lmo, d):
     rng = np.random.default_rng(d)
     B, H, cap, n_new = 3, 4, 48, 5
     cache = lmo.KVCache.empty(B, H, cap, d)
-    for t in (cache.k_codes, cache.v_codes, cache.k_meta, cache.v_meta):
-        t.view(torch.uint8).fill_(0xA5)
+    cache.kv.fill_(0xA5)
     host = oracle.new_cache(B, H, cap, d, fill=0xA5)
     k = (rng.standard_normal((B, H, n_new, d)) * 2).astype(np.float16)
     v = rng.standard_normal((B, H, n_new, d)).astype(np.float16)
@@ -162,7 +157,8 @@ CASES = [  # (B, Hkv, G, d, L, num_splits)
     (2, 3, 1, 64, 1, 0), (2, 3, 1, 128, 2, 0), (1, 2, 2, 128, 15, 0), (3, 2, 1, 128, 16, 0),
     (2, 4, 1, 128, 17, 0), (4, 12, 1, 64, 71, 0), (2, 2, 4, 128, 63, 0), (2, 2, 8, 128, 65, 1),
     (3, 5, 1, 128, 100, 3), (2, 2, 8, 64, 1000, 0), (1, 3, 1, 128, 1000, 7), (2, 1, 8, 128, 4090, 0),
-    (5, 7, 3, 128, 333, 0), (1, 1, 1, 128, 1, 4), (64, 8, 1, 128, 40, 0),
+    (5, 7, 3, 128, 333, 0), (1, 1, 1, 128, 1, 4), (64, 8, 1, 128, 40, 0), (3, 4, 2, 128, 517, 2),
+    (2, 3, 8, 128, 250, 4), (3, 2, 1, 64, 47, 2),
 ]
 
 

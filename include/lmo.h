@@ -148,11 +148,14 @@ size_t lmo_decode_attention_workspace_bytes(int32_t batch, int32_t kv_heads, int
  *               (1 <= len <= capacity, host-checked).
  * seq_lens_dev: optional device int32[batch]; L_b = min(seq_lens_dev[b],
  *               capacity); L_b <= 0 writes a zero output row.
- * num_splits  : 0 = auto (stream-K: the sequence blocks of all (b, kvh) pairs
- *               are divided evenly over the resident warps, partial results
- *               merged in-kernel by the last arriving warp);  k > 0 = each
- *               (b, kvh) pair is split into k contiguous parts (results then
- *               independent of batch composition).
+ * num_splits  : 0 = auto: "pair teams" (each (b, kvh) pair processed by a
+ *               team of 1, 2 or 4 warps of one CTA, combined on chip) when
+ *               there are enough pairs to fill the GPU, else "stream-K" (the
+ *               16-token blocks of all pairs divided evenly over the resident
+ *               warps; partial results merged in-kernel by the last arriving
+ *               warp).  1, 2, 4 = pair teams of that size; other k > 0 = each
+ *               pair split into k contiguous parts merged in-kernel.  With
+ *               k > 0 results do not depend on batch composition.
  * out         : [batch][q_heads][head_dim], LMO_F32 or LMO_F16.
  * q_heads/kv_heads must be in 1..8.
  * ------------------------------------------------------------------------- */
@@ -160,6 +163,23 @@ lmo_status lmo_decode_attention_q4(const lmo_kv_cache *cache, const void *q_f16,
                                    int32_t len, const int32_t *seq_lens_dev, float softmax_scale,
                                    int32_t num_splits, void *out, lmo_dtype out_dtype,
                                    void *workspace, size_t workspace_bytes, void *stream);
+
+/* ---------------------------------------------------------------------------
+ * A2+A3+A4 fused: one decode step of one layer -- append-quantize the new
+ * token's K/V (Eq 7) at slot L_b - 1, then attend over L_b tokens
+ * (the new token through its quantized form, reading 13).
+ * k_new_f16, v_new_f16 : [batch][kv_heads][head_dim] fp16 (the new token).
+ * len / seq_lens_dev give L_b as in lmo_decode_attention_q4 (new token
+ * included; L_b <= 0 appends nothing and writes a zero row).  Equivalent to
+ * lmo_kv_append_quant(pos = L_b - 1, n_new = 1) followed by
+ * lmo_decode_attention_q4 on the same stream, in one launch when the pair-team
+ * schedule is used (else two).  Other arguments as lmo_decode_attention_q4.
+ * ------------------------------------------------------------------------- */
+lmo_status lmo_decode_step_q4(const lmo_kv_cache *cache, const void *k_new_f16,
+                              const void *v_new_f16, const void *q_f16, int32_t q_heads,
+                              int32_t len, const int32_t *seq_lens_dev, float softmax_scale,
+                              int32_t num_splits, void *out, lmo_dtype out_dtype, void *workspace,
+                              size_t workspace_bytes, void *stream);
 
 /* Human-readable name of a status code (static string). */
 const char *lmo_status_string(lmo_status status);

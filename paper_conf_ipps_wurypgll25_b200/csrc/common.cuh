@@ -16,6 +16,7 @@ constexpr int kQMax = 15;    // 2^b - 1, b = 4
 // ------------------------------------------------------------ launch stats
 void note_launch();                         // lmo_abi.cu
 int device_sm_count();                      // cached per device
+bool pdl_enabled();                         // programmatic dependent launch on/off
 
 // ------------------------------------------------------- quantization math
 // One rounding chain, identical in every kernel that quantizes (K1, K2):

@@ -27,6 +27,7 @@
 //  * GQA: the query heads sharing a kv head are the MMA's head dimension, so
 //    a KV tile is read once for all of them (8 q heads per kv head cost the
 //    same HMMA count as 1).
+#include <cstdlib>
 #include <type_traits>
 
 #include "common.cuh"
@@ -83,6 +84,8 @@ struct AttnArgs {
     int out_f16;
     int *counters;            // [B*Hkv]
     float *partials;          // [slots][G][REC]
+    const __half *k_new;      // fused append (team mode): [B][Hkv][D] new token K, or nullptr
+    const __half *v_new;      //                            new token V
 };
 
 // ---------------------------------------------------------------- work map
@@ -159,8 +162,8 @@ struct SegIter {
         sn = n;
         wm.decode(x, b, kvh, blk, nb);
     }
-    // team mode: v = pair index, x0 = rank of this warp in its team
-    __device__ __noinline__ void team_seg(const WorkMap &wm) {
+    // team mode: v = pair index, x0 = rank of this warp in its team (inline: cheap)
+    __device__ __forceinline__ void team_seg(const WorkMap &wm) {
         if (v >= wm.B * wm.Hkv) {
             done = true;
             return;
@@ -174,11 +177,11 @@ struct SegIter {
         sx = wm.seq_start(b) + kvh * nb + lo;
         done = false;
     }
-    __device__ __noinline__ void begin_v(const WorkMap &wm) {
-        if (wm.T) {
-            team_seg(wm);
-            return;
-        }
+    __device__ __forceinline__ void begin_v(const WorkMap &wm) {
+        if (wm.T) team_seg(wm);
+        else begin_v_sk(wm);
+    }
+    __device__ __noinline__ void begin_v_sk(const WorkMap &wm) {
         while (v < wm.V) {
             x0 = wm.R(v);
             x1 = wm.R(v + 1);
@@ -203,12 +206,15 @@ struct SegIter {
         done = true;
     }
     // out of line: runs only at segment transitions, keeps the hot loop small (I-cache)
-    __device__ __noinline__ void next(const WorkMap &wm) {
+    __device__ __forceinline__ void next(const WorkMap &wm) {
         if (wm.T) {
             v += wm.n_teams;
             team_seg(wm);
-            return;
+        } else {
+            next_sk(wm);
         }
+    }
+    __device__ __noinline__ void next_sk(const WorkMap &wm) {
         if (phase == 0 && a < x1) {
             phase = 1;
             set_seg(wm, c, x1 - c);
@@ -223,7 +229,7 @@ struct SegIter {
             sn = nb;
         } else {
             v += wm.W;
-            begin_v(wm);
+            begin_v_sk(wm);
         }
     }
 };
@@ -376,6 +382,9 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int g = lane >> 2, t = lane & 3;
+    // Programmatic dependent launch: this grid may start while the previous kernel in
+    // the stream drains; wait here before touching any of its outputs (no-op otherwise).
+    asm volatile("griddepcontrol.wait;\n" ::: "memory");
 
     // ---- work map (identical in every CTA)
     if (a.lens) {
@@ -466,6 +475,45 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
         }
     };
 
+    // ---- fused append (A2) of each pair's new token at slot L_b - 1, by the warp that
+    // owns the pair's last block (team rank T-1) -- before any of its bulk copies, so
+    // its own TMA reads of that block see the quantized token (proxy fence below).
+    if (a.k_new && wms.T) {
+        const int T = wms.T, rank = gw % T;
+        if (rank == T - 1) {
+            const int lane8 = lane & 7, kvsel = lane / (8 * NG), grp = (lane >> 3) % NG;
+            const bool lane_ok = lane < 16 * NG;
+            for (int p = gw / T; p < a.B * a.Hkv; p += wms.n_teams) {
+                const int b = p / a.Hkv;
+                const int Lb = a.lens ? min(a.lens[b], a.cap) : a.len;
+                if (Lb < 1) continue;
+                const __half *src = (kvsel == 0 ? a.k_new : a.v_new) + (int64_t)p * D + grp * 64 + lane8 * 8;
+                uint4 xv = make_uint4(0, 0, 0, 0);
+                if (lane_ok) xv = *reinterpret_cast<const uint4 *>(src);
+                uint32_t mw;
+                const uint32_t w = quantize_group_lane8(xv, mw);
+                if (lane_ok) {
+                    uint8_t *row = const_cast<uint8_t *>(a.kv) + ((int64_t)p * a.cap + Lb - 1) * GG::ROW +
+                                   kvsel * (GG::RB + GG::MB);
+                    reinterpret_cast<uint32_t *>(row + grp * 32)[lane8] = w;
+                    if (lane8 == 0) reinterpret_cast<uint32_t *>(row + GG::RB)[grp] = mw;
+                }
+            }
+            asm volatile("fence.proxy.async.global;\n" ::: "memory");
+            __syncwarp();
+        }
+    }
+
+    // team mode: this warp's first pair is known -> start pulling its q rows into L2 now
+    if (wms.T && lane < a.G) {
+        const int p0 = gw / wms.T;
+        if (p0 < a.B * a.Hkv) {
+            const int b0 = p0 / a.Hkv, k0 = p0 - b0 * a.Hkv;
+            const char *qn = reinterpret_cast<const char *>(a.q + ((int64_t)b0 * a.Hq + k0 * a.G + lane) * D);
+#pragma unroll
+            for (int o = 0; o < D * 2; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(qn + o));
+        }
+    }
     if (lane == 0) {
         for (int s = 0; s < kStages; ++s) mbar_init(&wbar[s], 1);
         fence_mbar_init();
@@ -661,7 +709,10 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
             mb0 = max_over_g(mb0);
             mb1 = max_over_g(mb1);
             const float mn0 = fmaxf(m_run[0], mb0), mn1 = fmaxf(m_run[1], mb1);
-            if (__any_sync(0xffffffffu, (mn0 > m_run[0]) || (mn1 > m_run[1]))) {
+            // FULL stages rescale unconditionally (branch-free: one basic block with the
+            // next stage's K part, which ptxas can interleave); GEN stages skip it when
+            // no running max moved.
+            if (F || __any_sync(0xffffffffu, (mn0 > m_run[0]) || (mn1 > m_run[1]))) {
                 const float a0 = fast_exp2(m_run[0] - mn0), a1 = fast_exp2(m_run[1] - mn1);
                 m_run[0] = mn0;
                 m_run[1] = mn1;
@@ -825,30 +876,57 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
                 }
             }
             asm volatile("bar.sync %0, %1;\n" ::"r"(1 + warp / T), "r"(T * 32) : "memory");
-            if (gw % T == 0) {
+            // every warp of the team merges heads h = rank, rank + T, ...; all loads of a
+            // head are independent (one L2 round trip per head)
+            {
                 constexpr int DPL = D / 32;
-                for (int h = 0; h < a.G; ++h) {
+                const int rank = gw % T, gw0 = gw - rank;
+                const float *base = a.partials + (int64_t)(team_k & 1) * a.G * GG::REC;
+                for (int h = rank; h < a.G; h += T) {
+                    float mj[kWarps], lj[kWarps], oj[kWarps][DPL];
+#pragma unroll
+                    for (int j = 0; j < kWarps; ++j) {
+                        if (j < T) {
+                            const float *r = base + 2 * (int64_t)(gw0 + j) * a.G * GG::REC + h * GG::REC;
+                            mj[j] = __ldcg(r + D);
+                            lj[j] = __ldcg(r + D + 1);
+                            if constexpr (DPL == 4) {
+                                const float4 x = __ldcg(reinterpret_cast<const float4 *>(r) + lane);
+                                oj[j][0] = x.x; oj[j][1] = x.y; oj[j][2] = x.z; oj[j][3] = x.w;
+                            } else {
+#pragma unroll
+                                for (int i2 = 0; i2 < DPL; ++i2) oj[j][i2] = __ldcg(r + lane * DPL + i2);
+                            }
+                        }
+                    }
                     float M = NEG_INF;
-                    for (int j = 0; j < T; ++j)
-                        M = fmaxf(M, __ldcg(a.partials + (2 * (int64_t)(gw + j) + (team_k & 1)) * a.G * GG::REC + h * GG::REC + D));
+#pragma unroll
+                    for (int j = 0; j < kWarps; ++j) if (j < T) M = fmaxf(M, mj[j]);
                     if (M == NEG_INF) continue;          // empty sequence: zero row already written
                     float l = 0.f, o[DPL];
 #pragma unroll
                     for (int i2 = 0; i2 < DPL; ++i2) o[i2] = 0.f;
-                    for (int j = 0; j < T; ++j) {
-                        const float *r = a.partials + (2 * (int64_t)(gw + j) + (team_k & 1)) * a.G * GG::REC + h * GG::REC;
-                        const float w = exp2f(__ldcg(r + D) - M);
-                        l = fmaf(__ldcg(r + D + 1), w, l);
 #pragma unroll
-                        for (int i2 = 0; i2 < DPL; ++i2) o[i2] = fmaf(__ldcg(r + lane * DPL + i2), w, o[i2]);
+                    for (int j = 0; j < kWarps; ++j) {
+                        if (j < T) {
+                            const float w = fast_exp2(mj[j] - M);
+                            l = fmaf(lj[j], w, l);
+#pragma unroll
+                            for (int i2 = 0; i2 < DPL; ++i2) o[i2] = fmaf(oj[j][i2], w, o[i2]);
+                        }
                     }
                     const float il = 1.f / l;
                     const int64_t row = rowbase + h;
+                    if (a.out_f16) {
 #pragma unroll
-                    for (int i2 = 0; i2 < DPL; ++i2) {
-                        const int64_t off = row * D + lane * DPL + i2;
-                        if (a.out_f16) static_cast<__half *>(a.out)[off] = __float2half_rn(o[i2] * il);
-                        else static_cast<float *>(a.out)[off] = o[i2] * il;
+                        for (int i2 = 0; i2 < DPL; ++i2)
+                            static_cast<__half *>(a.out)[row * D + lane * DPL + i2] = __float2half_rn(o[i2] * il);
+                    } else if constexpr (DPL == 4) {
+                        reinterpret_cast<float4 *>(static_cast<float *>(a.out) + row * D)[lane] =
+                            make_float4(o[0] * il, o[1] * il, o[2] * il, o[3] * il);
+                    } else {
+#pragma unroll
+                        for (int i2 = 0; i2 < DPL; ++i2) static_cast<float *>(a.out)[row * D + lane * DPL + i2] = o[i2] * il;
                     }
                 }
             }
@@ -971,6 +1049,9 @@ extern "C" int lmo_debug_attn_profile(void *buf) {
 #endif
 
 // ---------------------------------------------------------------- host side
+cudaError_t launch_kv_append(const lmo_kv_cache &cache, const void *k_new, const void *v_new,
+                             int n_new, int pos0, const int32_t *pos_dev, cudaStream_t st,
+                             int pos_from_lens);
 template <int D>
 static size_t smem_bytes(int B_prefix) {
     return 128 + (size_t)kWarps * kStages * Geo<D>::STAGE + (B_prefix > 0 ? (B_prefix + 1) * sizeof(int) : 0);
@@ -1030,8 +1111,11 @@ static int choose_team(int64_t pairs, int64_t nb, int64_t warps) {
 
 cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq, int len,
                                     const int32_t *lens, float softmax_scale, int num_splits,
-                                    void *out, int out_f16, void *ws, cudaStream_t st) {
+                                    void *out, int out_f16, void *ws, cudaStream_t st,
+                                    const void *k_new, const void *v_new) {
     AttnArgs a;
+    a.k_new = static_cast<const __half *>(k_new);
+    a.v_new = static_cast<const __half *>(v_new);
     a.kv = c.kv;
     a.B = c.batch;
     a.Hkv = c.kv_heads;
@@ -1061,6 +1145,12 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     } else if (num_splits == 0 && !lens) {
         a.team = choose_team(pairs, nbu, (int64_t)max_ctas * kWarps);
     }
+    if (a.k_new && !a.team) {
+        // no pair teams (stream-K / fixed splits): append with its own kernel first
+        const cudaError_t e = launch_kv_append(c, k_new, v_new, 1, len - 1, lens, st, /*pos_from_lens=*/1);
+        if (e != cudaSuccess) return e;
+        a.k_new = a.v_new = nullptr;
+    }
     int64_t want_warps;
     if (a.team) {
         want_warps = pairs * a.team;
@@ -1073,10 +1163,21 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     int64_t ctas = (want_warps + kWarps - 1) / kWarps;
     if (ctas > max_ctas) ctas = max_ctas;
     if (ctas < 1) ctas = 1;
-    if (D == 64)
-        decode_attn_q4_kernel<64><<<(unsigned)ctas, kWarps * 32, smem_bytes<64>(Bp), st>>>(a);
-    else
-        decode_attn_q4_kernel<128><<<(unsigned)ctas, kWarps * 32, smem_bytes<128>(Bp), st>>>(a);
+    static const char *cap_env = getenv("LMO_ATTN_MAX_CTAS");   // tuning / experiments only
+    if (cap_env && atoi(cap_env) > 0 && ctas > atoi(cap_env)) ctas = atoi(cap_env);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)ctas);
+    cfg.blockDim = dim3(kWarps * 32);
+    cfg.dynamicSmemBytes = D == 64 ? smem_bytes<64>(Bp) : smem_bytes<128>(Bp);
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = D == 64 ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64>, a)
+                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128>, a);
+    if (e != cudaSuccess) return e;
     note_launch();
     return cudaGetLastError();
 }

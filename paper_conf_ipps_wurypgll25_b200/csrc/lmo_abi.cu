@@ -2,6 +2,7 @@
 // status codes, launch bookkeeping.  No exceptions cross the ABI; nothing is
 // launched or written when validation fails.
 #include <atomic>
+#include <cstdlib>
 #include <mutex>
 
 #include "common.cuh"
@@ -30,9 +31,20 @@ cudaError_t launch_quantize(const void *, int64_t, int64_t, int64_t, uint8_t *, 
 cudaError_t launch_dequantize(const uint8_t *, const lmo_qmeta *, int64_t, int64_t, int64_t,
                               void *, cudaStream_t);
 cudaError_t launch_kv_append(const lmo_kv_cache &, const void *, const void *, int, int,
-                             const int32_t *, cudaStream_t);
+                             const int32_t *, cudaStream_t, int pos_from_lens);
 cudaError_t launch_decode_attention(const lmo_kv_cache &, const void *, int, int, const int32_t *,
-                                    float, int, void *, int, void *, cudaStream_t);
+                                    float, int, void *, int, void *, cudaStream_t, const void *,
+                                    const void *);
+
+// Programmatic dependent launch for the hot-path kernels (LMO_PDL=0 disables).
+bool pdl_enabled() {
+    static int v = -1;
+    if (v < 0) {
+        const char *e = getenv("LMO_PDL");
+        v = (e && e[0] == '0') ? 0 : 1;
+    }
+    return v == 1;
+}
 cudaError_t launch_gen_fill(void *, int, int, int, int, uint64_t, int, int, int, int, int, int,
                             cudaStream_t);
 size_t attn_workspace_bytes(int B, int Hkv, int Hq, int D, int num_splits);
@@ -89,7 +101,7 @@ lmo_status lmo_kv_append_quant(const lmo_kv_cache *cache, const void *k_new, con
     if (!pos_dev && (pos0 < 0 || (int64_t)pos0 + n_new > cache->capacity)) return LMO_ERR_SHAPE;
     if (!aligned16(k_new) || !aligned16(v_new)) return LMO_ERR_ALIGN;
     return cuda_status(launch_kv_append(*cache, k_new, v_new, n_new, pos0, pos_dev,
-                                        static_cast<cudaStream_t>(stream)));
+                                        static_cast<cudaStream_t>(stream), 0));
 }
 
 size_t lmo_decode_attention_workspace_bytes(int32_t batch, int32_t kv_heads, int32_t q_heads,
@@ -100,10 +112,10 @@ size_t lmo_decode_attention_workspace_bytes(int32_t batch, int32_t kv_heads, int
     return attn_workspace_bytes(batch, kv_heads, q_heads, head_dim, num_splits);
 }
 
-lmo_status lmo_decode_attention_q4(const lmo_kv_cache *cache, const void *q, int32_t q_heads,
-                                   int32_t len, const int32_t *seq_lens_dev, float softmax_scale,
-                                   int32_t num_splits, void *out, lmo_dtype out_dtype,
-                                   void *workspace, size_t workspace_bytes, void *stream) {
+static lmo_status check_attention(const lmo_kv_cache *cache, const void *q, int32_t q_heads,
+                                  int32_t len, const int32_t *seq_lens_dev, int32_t num_splits,
+                                  void *out, lmo_dtype out_dtype, void *workspace,
+                                  size_t workspace_bytes) {
     lmo_status s = check_cache(cache);
     if (s != LMO_OK) return s;
     if (!q || !out) return LMO_ERR_NULL;
@@ -113,15 +125,45 @@ lmo_status lmo_decode_attention_q4(const lmo_kv_cache *cache, const void *q, int
     if (out_dtype != LMO_F16 && out_dtype != LMO_F32) return LMO_ERR_UNSUPPORTED;
     if (!seq_lens_dev && (len < 1 || len > cache->capacity)) return LMO_ERR_SHAPE;
     if (seq_lens_dev && cache->batch > 1024) return LMO_ERR_UNSUPPORTED;
+    if ((int64_t)cache->batch * cache->kv_heads * ((int64_t)cache->capacity / 16) > (1LL << 30))
+        return LMO_ERR_SHAPE;
     if (!aligned16(q) || !aligned16(out)) return LMO_ERR_ALIGN;
     const size_t need = attn_workspace_bytes(cache->batch, cache->kv_heads, q_heads,
                                              cache->head_dim, num_splits);
     if (!workspace || workspace_bytes < need) return LMO_ERR_WORKSPACE;
     if (!aligned16(workspace)) return LMO_ERR_ALIGN;
+    return LMO_OK;
+}
+
+lmo_status lmo_decode_attention_q4(const lmo_kv_cache *cache, const void *q, int32_t q_heads,
+                                   int32_t len, const int32_t *seq_lens_dev, float softmax_scale,
+                                   int32_t num_splits, void *out, lmo_dtype out_dtype,
+                                   void *workspace, size_t workspace_bytes, void *stream) {
+    const lmo_status s = check_attention(cache, q, q_heads, len, seq_lens_dev, num_splits, out,
+                                         out_dtype, workspace, workspace_bytes);
+    if (s != LMO_OK) return s;
     return cuda_status(launch_decode_attention(*cache, q, q_heads, len, seq_lens_dev,
                                                softmax_scale, num_splits, out,
                                                out_dtype == LMO_F16 ? 1 : 0, workspace,
-                                               static_cast<cudaStream_t>(stream)));
+                                               static_cast<cudaStream_t>(stream), nullptr,
+                                               nullptr));
+}
+
+lmo_status lmo_decode_step_q4(const lmo_kv_cache *cache, const void *k_new_f16,
+                              const void *v_new_f16, const void *q, int32_t q_heads, int32_t len,
+                              const int32_t *seq_lens_dev, float softmax_scale, int32_t num_splits,
+                              void *out, lmo_dtype out_dtype, void *workspace,
+                              size_t workspace_bytes, void *stream) {
+    const lmo_status s = check_attention(cache, q, q_heads, len, seq_lens_dev, num_splits, out,
+                                         out_dtype, workspace, workspace_bytes);
+    if (s != LMO_OK) return s;
+    if (!k_new_f16 || !v_new_f16) return LMO_ERR_NULL;
+    if (!aligned16(k_new_f16) || !aligned16(v_new_f16)) return LMO_ERR_ALIGN;
+    return cuda_status(launch_decode_attention(*cache, q, q_heads, len, seq_lens_dev,
+                                               softmax_scale, num_splits, out,
+                                               out_dtype == LMO_F16 ? 1 : 0, workspace,
+                                               static_cast<cudaStream_t>(stream), k_new_f16,
+                                               v_new_f16));
 }
 
 const char *lmo_status_string(lmo_status st) {

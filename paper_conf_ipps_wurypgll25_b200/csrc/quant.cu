@@ -77,7 +77,9 @@ __global__ void __launch_bounds__(256) kv_append_kernel(lmo_kv_cache cache,
                                                         const __half *__restrict__ k_new,
                                                         const __half *__restrict__ v_new,
                                                         int n_new, int pos0,
-                                                        const int32_t *__restrict__ pos_dev) {
+                                                        const int32_t *__restrict__ pos_dev,
+                                                        int pos_from_lens) {
+    asm volatile("griddepcontrol.wait;\n" ::: "memory");   // PDL: inputs of earlier kernels
     const int d = cache.head_dim;
     const int gpr = d / kGroup;
     const int lane8 = threadIdx.x & 7;
@@ -92,7 +94,8 @@ __global__ void __launch_bounds__(256) kv_append_kernel(lmo_kv_cache cache,
     const int t = (int)(r % n_new);
     const int64_t bh = r / n_new;
     const int b = (int)(bh / cache.kv_heads);
-    const int pos = pos_dev ? pos_dev[b] : pos0;
+    int pos = pos_dev ? pos_dev[b] : pos0;
+    if (pos_dev && pos_from_lens) pos = min(pos, cache.capacity) - 1;   // new token at L_b - 1
     if (pos < 0 || pos + n_new > cache.capacity) valid = false;
     const __half *src = (kv == 0 ? k_new : v_new) + r * d + grp * kGroup + lane8 * 8;
     uint4 xv = make_uint4(0, 0, 0, 0);
@@ -196,15 +199,26 @@ cudaError_t launch_dequantize(const uint8_t *codes, const lmo_qmeta *meta, int64
 }
 
 cudaError_t launch_kv_append(const lmo_kv_cache &cache, const void *k_new, const void *v_new,
-                             int n_new, int pos0, const int32_t *pos_dev, cudaStream_t st) {
+                             int n_new, int pos0, const int32_t *pos_dev, cudaStream_t st,
+                             int pos_from_lens) {
     const int64_t groups =
         2LL * cache.batch * cache.kv_heads * n_new * (cache.head_dim / kGroup);
     const int64_t blocks = (groups + 31) / 32;
-    kv_append_kernel<<<(unsigned)blocks, 256, 0, st>>>(cache, static_cast<const __half *>(k_new),
-                                                       static_cast<const __half *>(v_new), n_new,
-                                                       pos0, pos_dev);
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)blocks);
+    cfg.blockDim = dim3(256);
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    const cudaError_t e = cudaLaunchKernelEx(&cfg, kv_append_kernel, cache,
+                                             static_cast<const __half *>(k_new),
+                                             static_cast<const __half *>(v_new), n_new, pos0, pos_dev,
+                                             pos_from_lens);
     note_launch();
-    return cudaGetLastError();
+    return e != cudaSuccess ? e : cudaGetLastError();
 }
 
 }  // namespace lmo

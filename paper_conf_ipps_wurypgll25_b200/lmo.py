@@ -46,6 +46,8 @@ def _load():
         "lmo_decode_attention_q4": [ctypes.POINTER(lmo_kv_cache), P, i32, i32, P, ctypes.c_float,
                                     i32, P, ctypes.c_int, P, ctypes.c_size_t, P],
         "lmo_gen_fill_f16": [P, i32, i32, i32, i32, u64, i32, i32, i32, i32, i32, i32, P],
+        "lmo_decode_step_q4": [ctypes.POINTER(lmo_kv_cache), P, P, P, i32, i32, P, ctypes.c_float,
+                               i32, P, ctypes.c_int, P, ctypes.c_size_t, P],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -68,7 +70,8 @@ _lib = _load()
 LIB_PATH = _build.LIB
 EXPORTS = ["lmo_quantize_groupwise", "lmo_dequantize_groupwise", "lmo_kv_append_quant",
            "lmo_kv_row_bytes",
-           "lmo_decode_attention_workspace_bytes", "lmo_decode_attention_q4", "lmo_status_string",
+           "lmo_decode_attention_workspace_bytes", "lmo_decode_attention_q4", "lmo_decode_step_q4",
+           "lmo_status_string",
            "lmo_gen_fill_f16", "lmo_launch_count", "lmo_version"]
 
 
@@ -229,6 +232,30 @@ def lmo_decode_attention_q4(cache: KVCache, q: torch.Tensor, length: int = 0,
                                         float(softmax_scale), num_splits, _ptr(out), dt,
                                         _ptr(workspace), workspace.numel(), _stream(stream)),
            "lmo_decode_attention_q4")
+    return out
+
+
+def lmo_decode_step_q4(cache: KVCache, k_new: torch.Tensor, v_new: torch.Tensor, q: torch.Tensor,
+                       length: int = 0, seq_lens: torch.Tensor | None = None,
+                       softmax_scale: float | None = None, num_splits: int = 0,
+                       out: torch.Tensor | None = None, out_dtype: torch.dtype = torch.float32,
+                       workspace: torch.Tensor | None = None, stream=None, abi=None) -> torch.Tensor:
+    """One decode step of one layer: append the new token's K/V ([B][Hkv][d] or
+    [B][Hkv][1][d]) at slot L-1, then attention over L (A2+A3+A4 fused)."""
+    B, Hq, d = q.shape
+    if softmax_scale is None:
+        softmax_scale = 1.0 / math.sqrt(d)
+    if out is None:
+        out = torch.empty((B, Hq, d), dtype=out_dtype, device=q.device)
+    if workspace is None:
+        workspace = attention_workspace(cache.batch, cache.kv_heads, Hq, cache.head_dim,
+                                        num_splits, q.device)
+    dt = LMO_F16 if out.dtype == torch.float16 else LMO_F32
+    c = abi if abi is not None else cache.abi()
+    _check(_lib.lmo_decode_step_q4(ctypes.byref(c), _ptr(k_new), _ptr(v_new), _ptr(q), Hq, length,
+                                   _ptr(seq_lens), float(softmax_scale), num_splits, _ptr(out), dt,
+                                   _ptr(workspace), workspace.numel(), _stream(stream)),
+           "lmo_decode_step_q4")
     return out
 
 

@@ -260,3 +260,68 @@ def test_full_size_sampled_rows(lmo, key):
         ref = oracle.decode_attention_q4(one, qh, L)
         err = normwise_err(out[b, kvh * G:(kvh + 1) * G].cpu().numpy(), ref[0])
         assert err.max() <= TOL, (b, kvh, err.max())
+
+
+# ------------------------------------------ fused decode step (A2+A3+A4) ----
+
+@pytest.mark.parametrize("B,Hkv,G,d,L,ns", [(4, 6, 1, 128, 300, 0), (2, 2, 8, 128, 129, 0),
+                                            (3, 4, 2, 64, 77, 2), (2, 3, 1, 128, 40, 4),
+                                            (2, 2, 4, 128, 200, 3), (1, 2, 1, 128, 1, 0)])
+def test_decode_step_fused_append(lmo, B, Hkv, G, d, L, ns):
+    """lmo_decode_step_q4 == append(new token at L-1) then attention over L, for the
+    team schedule (one launch) and the stream-K fallback (two launches)."""
+    seed = 31 + L
+    cap = L + 7
+    kf = torch.empty((B, Hkv, L, d), dtype=torch.float16, device="cuda")
+    vf = torch.empty_like(kf)
+    lmo.lmo_gen_fill_f16(kf, seed, I.STREAM_K, 0, 0, 0, 0)
+    lmo.lmo_gen_fill_f16(vf, seed, I.STREAM_V, 0, 0, 0, 0)
+    cache = lmo.KVCache.empty(B, Hkv, cap, d)
+    cache.kv.fill_(0x7B)
+    if L > 1:
+        lmo.lmo_kv_append_quant(cache, kf[:, :, :L - 1].contiguous(), vf[:, :, :L - 1].contiguous(), 0)
+    q = torch.empty((B, Hkv * G, 1, d), dtype=torch.float16, device="cuda")
+    lmo.lmo_gen_fill_f16(q, seed, I.STREAM_Q, 0, 0, 0, 0, group=G)
+    q = q.view(B, Hkv * G, d)
+    out = lmo.lmo_decode_step_q4(cache, kf[:, :, L - 1].contiguous(), vf[:, :, L - 1].contiguous(),
+                                 q, L, num_splits=ns)
+    torch.cuda.synchronize()
+    host = oracle.new_cache(B, Hkv, cache.capacity, d)
+    oracle.kv_append_quant(host, kf.cpu().numpy(), vf.cpu().numpy(), 0)
+    got = cache_to_host(cache)
+    for key in host:
+        assert np.array_equal(got[key][:, :, :L], host[key][:, :, :L]), key
+    ref = oracle.decode_attention_q4(host, q.cpu().numpy(), L, nthreads=8)
+    assert normwise_err(out.cpu().numpy(), ref).max() <= TOL
+
+
+def test_decode_step_per_sequence_lengths(lmo):
+    B, Hkv, G, d, cap = 5, 3, 2, 128, 208
+    lens = np.array([200, 1, 0, 65, 129], np.int32)
+    kf = torch.empty((B, Hkv, cap, d), dtype=torch.float16, device="cuda")
+    vf = torch.empty_like(kf)
+    lmo.lmo_gen_fill_f16(kf, 9, I.STREAM_K, 0, 0, 0, 0)
+    lmo.lmo_gen_fill_f16(vf, 9, I.STREAM_V, 0, 0, 0, 0)
+    cache = lmo.KVCache.empty(B, Hkv, cap, d)
+    lmo.lmo_kv_append_quant(cache, kf, vf, 0)               # whole capacity (stale beyond L)
+    kn = torch.empty((B, Hkv, 1, d), dtype=torch.float16, device="cuda")
+    vn = torch.empty_like(kn)
+    lmo.lmo_gen_fill_f16(kn, 10, I.STREAM_K, 0, 0, 0, 0)
+    lmo.lmo_gen_fill_f16(vn, 10, I.STREAM_V, 0, 0, 0, 0)
+    q = torch.empty((B, Hkv * G, 1, d), dtype=torch.float16, device="cuda")
+    lmo.lmo_gen_fill_f16(q, 9, I.STREAM_Q, 0, 0, 0, 0, group=G)
+    q = q.view(B, Hkv * G, d)
+    out = lmo.lmo_decode_step_q4(cache, kn, vn, q, 0, seq_lens=dev(lens))
+    torch.cuda.synchronize()
+    kh, vh = kf.cpu().numpy().copy(), vf.cpu().numpy().copy()
+    for b in range(B):
+        if lens[b] > 0:
+            kh[b, :, lens[b] - 1] = kn.cpu().numpy()[b, :, 0]
+            vh[b, :, lens[b] - 1] = vn.cpu().numpy()[b, :, 0]
+    host = oracle.new_cache(B, Hkv, cache.capacity, d)
+    oracle.kv_append_quant(host, kh, vh, 0)
+    ref = oracle.decode_attention_q4(host, q.cpu().numpy(), np.maximum(lens, 1), nthreads=8)
+    o = out.cpu().numpy()
+    keep = lens > 0
+    assert np.all(o[~keep] == 0)
+    assert normwise_err(o[keep], ref[keep]).max() <= TOL

@@ -369,7 +369,7 @@ struct KState {       // per-stage scores handed from the K part to the V part
     float z[kSub][2][2];
 };
 
-template <int D>
+template <int D, bool MHA>
 __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q4_kernel(const AttnArgs a) {
     using GG = Geo<D>;
     constexpr int NG = GG::NG;
@@ -585,8 +585,9 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
 #pragma unroll
                 for (int grp = 0; grp < NG; ++grp) {
                     uint4 q0 = make_uint4(0, 0, 0, 0), q1 = q0;
-                    if (g < a.G) {
-                        const __half *qp = a.q + (((int64_t)b * a.Hq + kvh * a.G + g) * D + grp * 64 + 16 * t);
+                    // MHA: q replicated into all 8 columns -> every lane's C holds real scores
+                    if (MHA || g < a.G) {
+                        const __half *qp = a.q + (((int64_t)b * a.Hq + kvh * a.G + (MHA ? 0 : g)) * D + grp * 64 + 16 * t);
                         q0 = *reinterpret_cast<const uint4 *>(qp);
                         q1 = *reinterpret_cast<const uint4 *>(qp + 8);
                     }
@@ -651,6 +652,46 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
             constexpr bool F = decltype(full)::value;
             const uint32_t st = sl * GG::STAGE;
             const int nsub = F ? kSub : min(kSub, seg_n - jb);
+            if constexpr (MHA) {
+                // every lane scores ONE token of the stage: sub-block ls = t>>1, row g (+8 if t odd)
+                const int ls = t >> 1, hi = t & 1;
+                float S[NG];
+#pragma unroll
+                for (int grp = 0; grp < NG; ++grp) S[grp] = 0.f;
+#pragma unroll
+                for (int s = 0; s < kSub; ++s) {
+                    if (s < nsub) {
+                        const uint32_t ss = st + s * dSC;
+#pragma unroll
+                        for (int grp = 0; grp < NG; ++grp) {
+                            const uint2 w0 = lds64(ss + offK0 + grp * 32);
+                            const uint2 w1 = lds64(ss + offK0 + dK1 + grp * 32);
+                            uint32_t u0[8], u1[8];
+                            unpack_k(w0.x, u0);
+                            unpack_k(w0.y, u0 + 4);
+                            unpack_k(w1.x, u1);
+                            unpack_k(w1.y, u1 + 4);
+                            float c[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+                            for (int kbl = 0; kbl < 4; ++kbl)
+                                mma_16816(c, u0[2 * kbl], u1[2 * kbl], u0[2 * kbl + 1], u1[2 * kbl + 1],
+                                          qf[grp][kbl][0], qf[grp][kbl][1]);
+                            if (s == ls) S[grp] = hi ? c[2] : c[0];
+                        }
+                    }
+                }
+                const int row = hi ? tk1 : tk0;
+                const uint2 km = load_meta<NG>(ring_u32 + st + ls * dSM + row * GG::ROW + GG::OKM);
+                float z = 0.f;
+#pragma unroll
+                for (int grp = 0; grp < NG; ++grp) {
+                    const float2 f = meta_f2(grp == 0 ? km.x : km.y);
+                    z = fmaf(S[grp], f.y * zs24, fmaf(f.x * zs, qs[grp][0], z));
+                }
+                const int tokbase = (blk0 + jb + ls) * kBlk;
+                if (!F && (ls >= nsub || tokbase + row >= L)) z = NEG_INF;
+                ks.z[0][0][0] = z;
+            } else {
 #pragma unroll
             for (int s = 0; s < kSub; ++s) {
                 if (s < nsub) {
@@ -696,6 +737,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
                     ks.z[s][0][0] = ks.z[s][0][1] = ks.z[s][1][0] = ks.z[s][1][1] = NEG_INF;
                 }
             }
+            }
         };
 
         // softmax + V part of one stage, then hand the slot back to the producer
@@ -704,6 +746,74 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
             const uint32_t st = sl * GG::STAGE;
             const int nsub = F ? kSub : min(kSub, seg_n - jb);
             const bool tail = !F && (blk0 + jb + kSub) * kBlk > L;
+            if constexpr (MHA) {
+                // ---- one token per lane: warp-wide running max, p, V meta, w = p*scale
+                const int ls = t >> 1, hi = t & 1;
+                const int row = hi ? tk1 : tk0;
+                const float z = ks.z[0][0][0];
+                float mb = z;
+#pragma unroll
+                for (int off = 16; off > 0; off >>= 1) mb = fmaxf(mb, __shfl_xor_sync(0xffffffffu, mb, off));
+                if (mb > m_run[0]) {                          // warp-uniform
+                    const float a0 = fast_exp2(m_run[0] - mb);
+                    m_run[0] = mb;
+                    l_run[0] *= a0;
+#pragma unroll
+                    for (int grp = 0; grp < NG; ++grp) pm[0][grp] *= a0;
+#pragma unroll
+                    for (int i = 0; i < NG * 4; ++i) {
+                        acc[i][0] *= a0;
+                        acc[i][1] *= a0;
+                        acc[i][2] *= a0;
+                        acc[i][3] *= a0;
+                    }
+                }
+                const float p = fast_exp2(z - m_run[0]);
+                l_run[0] += p;
+                const uint2 vmw = load_meta<NG>(ring_u32 + st + ls * dSM + row * GG::ROW + GG::OVM);
+                float w[2] = {0.f, 0.f};
+#pragma unroll
+                for (int grp = 0; grp < NG; ++grp) {
+                    float2 f = meta_f2(grp == 0 ? vmw.x : vmw.y);
+                    if (!F && z == NEG_INF) f = make_float2(0.f, 0.f);     // stale meta of masked slots
+                    pm[0][grp] = fmaf(p, f.x, pm[0][grp]);
+                    w[grp] = p * f.y;
+                }
+                const uint32_t xw = pack_half2(w[0], w[1]);           // (group 0, group 1)
+#pragma unroll
+                for (int s = 0; s < kSub; ++s) {
+                    if (s < nsub) {
+                        // B = P^T: k = 2t, 2t+1 (rows 2t, 2t+1) and 2t+8, 2t+9 (rows +8), any column
+                        const uint32_t x0 = __shfl_sync(0xffffffffu, xw, 8 * t + 2 * s);
+                        const uint32_t x1 = __shfl_sync(0xffffffffu, xw, 8 * t + 4 + 2 * s);
+                        const uint32_t x2 = __shfl_sync(0xffffffffu, xw, 8 * t + 2 * s + 1);
+                        const uint32_t x3 = __shfl_sync(0xffffffffu, xw, 8 * t + 5 + 2 * s);
+                        const uint32_t ss = st + s * dSC;
+#pragma unroll
+                        for (int grp = 0; grp < NG; ++grp) {
+                            const uint32_t sel = grp == 0 ? 0x5410u : 0x7632u;
+                            const uint32_t bp0 = prmt(x0, x1, sel), bp1 = prmt(x2, x3, sel);
+                            const uint32_t wa0 = lds32(ss + offVa0 + grp * 32);
+                            const uint32_t wb0 = lds32(ss + offVb0 + grp * 32);
+                            const uint32_t wa1 = lds32(ss + offVa0 + dK1 + grp * 32);
+                            const uint32_t wb1 = lds32(ss + offVb0 + dK1 + grp * 32);
+                            uint32_t j0[8], j1[8];
+                            unpack_v(wa0, wb0, j0);
+                            unpack_v(wa1, wb1, j1);
+#pragma unroll
+                            for (int mbl = 0; mbl < 4; ++mbl)
+                                mma_16816(acc[grp * 4 + mbl], j0[2 * mbl], j0[2 * mbl + 1], j1[2 * mbl],
+                                          j1[2 * mbl + 1], bp0, bp1);
+                        }
+                    }
+                }
+                __syncwarp();
+                if (lane == 0 && !ctl.pc.done) issue(sl);
+#if LMO_ATTN_PROFILE
+                ++prof_st;
+#endif
+                return;
+            }
             float mb0 = fmaxf(fmaxf(ks.z[0][0][0], ks.z[0][1][0]), fmaxf(ks.z[kSub - 1][0][0], ks.z[kSub - 1][1][0]));
             float mb1 = fmaxf(fmaxf(ks.z[0][0][1], ks.z[0][1][1]), fmaxf(ks.z[kSub - 1][0][1], ks.z[kSub - 1][1][1]));
             mb0 = max_over_g(mb0);
@@ -835,11 +945,25 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
         // ------------------------------------------------ segment end
         // heads 2t+e: reduce l and Pm over the 8 g-lanes; O = 2^24 acc(row g) / 2^20 acc(row g+8) + Pm
         float lt[2], pmt[2][NG];
+        if constexpr (MHA) {      // per-lane tokens: full-warp sums; head 0 only
+            float l = l_run[0];
+#pragma unroll
+            for (int off = 16; off > 0; off >>= 1) l += __shfl_xor_sync(0xffffffffu, l, off);
+            lt[0] = lt[1] = l;
+#pragma unroll
+            for (int grp = 0; grp < NG; ++grp) {
+                float v = pm[0][grp];
+#pragma unroll
+                for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(0xffffffffu, v, off);
+                pmt[0][grp] = pmt[1][grp] = v;
+            }
+        } else {
 #pragma unroll
         for (int e = 0; e < 2; ++e) {
             lt[e] = sum_over_g(l_run[e]);
 #pragma unroll
             for (int grp = 0; grp < NG; ++grp) pmt[e][grp] = sum_over_g(pm[e][grp]);
+        }
         }
         float vo[2][NG][8];
 #pragma unroll
@@ -1058,18 +1182,22 @@ static size_t smem_bytes(int B_prefix) {
 }
 
 template <int D>
-static int ctas_per_sm(int B_prefix) {
+static int ctas_per_sm(int B_prefix) {   // (MHA and GQA variants have the same resources)
     static int occ[64][2] = {{0}};
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev < 0 || dev >= 64) dev = 0;
     const int mode = B_prefix > 0 ? 1 : 0;
     if (occ[dev][mode] == 0) {
-        cudaFuncSetAttribute(decode_attn_q4_kernel<D>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)smem_bytes<D>(kMaxBatchSmem));
-        int n = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, decode_attn_q4_kernel<D>, kWarps * 32,
+        for (int m = 0; m < 2; ++m)
+            cudaFuncSetAttribute(m ? decode_attn_q4_kernel<D, true> : decode_attn_q4_kernel<D, false>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes<D>(kMaxBatchSmem));
+        int n = 0, n1 = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n1, decode_attn_q4_kernel<D, true>, kWarps * 32,
                                                       smem_bytes<D>(mode ? kMaxBatchSmem : 0));
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, decode_attn_q4_kernel<D, false>, kWarps * 32,
+                                                      smem_bytes<D>(mode ? kMaxBatchSmem : 0));
+        if (n1 < n) n = n1;
         occ[dev][mode] = n > 0 ? n : 1;
     }
     return occ[dev][mode];
@@ -1175,8 +1303,11 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
-    cudaError_t e = D == 64 ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64>, a)
-                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128>, a);
+    const bool mha = a.G == 1;
+    cudaError_t e = D == 64 ? (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, true>, a)
+                                   : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false>, a))
+                            : (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, true>, a)
+                                   : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, false>, a));
     if (e != cudaSuccess) return e;
     note_launch();
     return cudaGetLastError();

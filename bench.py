@@ -213,7 +213,8 @@ def run_ours(args):
     w = C.CONFIGS[args.config]
     seed = I.seed_for_config(w.index)
     B, Hkv, Hq, d, G, s = w.batch, w.kv_heads, w.q_heads, w.head_dim, w.group_ratio, w.prompt
-    b_off = rank * B                      # global batch offset (weak scaling)
+    from paper_conf_ipps_wurypgll25_b200 import dist as D
+    b_off, _ = D.shard(rank, world, B)    # global batch offset (weak scaling, no hot-path collective)
     nl = w.layers
     steps_total = args.warmup + args.steps
     # Timed decode steps are spread evenly over the whole generation t = 1..n-1
@@ -303,11 +304,7 @@ def run_ours(args):
         torch.cuda.synchronize()
 
     def reduce_max(x: float) -> float:
-        if world == 1:
-            return x
-        tt = torch.tensor([x], dtype=torch.float64, device=dev)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        return float(tt.item())
+        return D.max_over_ranks(x, device=dev)
 
     # ---- warm-up + timed steps (device-resident inputs).  The clock sampler runs
     # across a ~0.5 s load window that ends with the timed region (warm-up steps

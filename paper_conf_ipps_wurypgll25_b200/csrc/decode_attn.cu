@@ -483,7 +483,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
         if (rank == T - 1) {
             const int lane8 = lane & 7, kvsel = lane / (8 * NG), grp = (lane >> 3) % NG;
             const bool lane_ok = lane < 16 * NG;
-            for (int p = gw / T; p < a.B * a.Hkv; p += wms.n_teams) {
+            for (int p = (warp / T) * gridDim.x + blockIdx.x; p < a.B * a.Hkv; p += wms.n_teams) {
                 const int b = p / a.Hkv;
                 const int Lb = a.lens ? min(a.lens[b], a.cap) : a.len;
                 if (Lb < 1) continue;
@@ -506,7 +506,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
 
     // team mode: this warp's first pair is known -> start pulling its q rows into L2 now
     if (wms.T && lane < a.G) {
-        const int p0 = gw / wms.T;
+        const int p0 = (warp / wms.T) * gridDim.x + blockIdx.x;
         if (p0 < a.B * a.Hkv) {
             const int b0 = p0 / a.Hkv, k0 = p0 - b0 * a.Hkv;
             const char *qn = reinterpret_cast<const char *>(a.q + ((int64_t)b0 * a.Hq + k0 * a.G + lane) * D);
@@ -518,8 +518,10 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
         for (int s = 0; s < kStages; ++s) mbar_init(&wbar[s], 1);
         fence_mbar_init();
         if (wms.T) {
-            ctl.cc.v = gw / wms.T;           // team id = first pair
-            ctl.cc.x0 = gw % wms.T;          // rank in team
+            // team ids interleaved across CTAs (tau = team-in-CTA * grid + CTA): the busy
+            // teams spread evenly over the SMs when there are fewer pairs than teams
+            ctl.cc.v = (warp / wms.T) * gridDim.x + blockIdx.x;   // team id = first pair
+            ctl.cc.x0 = warp % wms.T;                             // rank in team
         } else {
             ctl.cc.v = gw;
         }
@@ -1216,25 +1218,17 @@ size_t attn_workspace_bytes(int B, int Hkv, int Hq, int D, int num_splits) {
     return counters + slots * G * (D + 4) * sizeof(float);
 }
 
-// Work distribution (uniform length): pair teams of T in {1, 2, 4} warps, or
-// stream-K when there are too few pairs to fill the resident warps.  Cost in
-// units of one stage (32 tokens) of one warp, with a per-pair overhead.
-static int choose_team(int64_t pairs, int64_t nb, int64_t warps) {
-    const int64_t S = (nb + kSub - 1) / kSub;
-    double best = 1e30;
-    int bestT = 0;
-    for (int T = 1; T <= kWarps; T *= 2) {
-        const int64_t teams = warps / T;
-        const int64_t rounds = (pairs + teams - 1) / teams;
-        const double per = (double)((((nb + T - 1) / T) + kSub - 1) / kSub) + (T == 1 ? 1.0 : 2.0);
-        const double cost = rounds * per;
-        if (cost < best) {
-            best = cost;
-            bestT = T;
-        }
-    }
-    const double sk = (double)pairs * S / (double)warps + 4.0;   // stream-K: balanced + merge overhead
-    return sk < 0.9 * best ? 0 : bestT;
+// Work distribution: persistent pair teams -- each (b, kv-head) pair is
+// processed by a team of T warps of one CTA; a warp's producer runs ahead
+// across the pairs it processes, so a pair boundary costs no pipeline bubble.
+// T = 1 when the pairs can keep a fair share of the resident warps busy, else
+// 2 or 4 (few pairs: a pair's blocks are split over more warps).  Stream-K
+// (balanced block ranges with a global last-arriver merge) is kept for
+// explicit use; measured slower than teams on every BASELINE config.
+static int choose_team(int64_t pairs, int64_t warps) {
+    for (int T = 1; T < kWarps; T *= 2)
+        if ((double)pairs * T >= 0.35 * (double)warps) return T;
+    return kWarps;
 }
 
 cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq, int len,
@@ -1270,8 +1264,11 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     if (num_splits == 1 || num_splits == 2 || num_splits == 4) {
         a.team = num_splits;                  // explicit team size (batch-independent results)
         a.num_splits = 0;
-    } else if (num_splits == 0 && !lens) {
-        a.team = choose_team(pairs, nbu, (int64_t)max_ctas * kWarps);
+    } else if (num_splits == 0) {
+        a.team = choose_team(pairs, (int64_t)max_ctas * kWarps);
+        static const char *sched = getenv("LMO_ATTN_SCHED");   // experiments: streamk | team1|2|4
+        if (sched && sched[0] == 's') a.team = 0;
+        if (sched && sched[0] == 't') a.team = atoi(sched + 4);
     }
     if (a.k_new && !a.team) {
         // no pair teams (stream-K / fixed splits): append with its own kernel first
@@ -1281,7 +1278,7 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     }
     int64_t want_warps;
     if (a.team) {
-        want_warps = pairs * a.team;
+        want_warps = (int64_t)max_ctas * kWarps;          // all CTAs; idle teams exit at once
     } else if (lens) {
         want_warps = (int64_t)max_ctas * kWarps;
     } else {

@@ -44,6 +44,7 @@ def parse():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--splits", type=int, default=0, help="num_splits (0 = stream-K auto)")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-early", action="store_true", help="disable LMO_STEP_CACHE_STABLE")
     p.add_argument("--cpu-sample-seconds", type=float, default=10.0)
     return p.parse_args()
 
@@ -273,7 +274,8 @@ def run_ours(args):
             if append and attn:
                 lmo.lmo_decode_step_q4(caches[l], kbuf[t][l], vbuf[t][l], qbuf[t][l].view(B, Hq, d),
                                        s + t, softmax_scale=sigma, num_splits=args.splits,
-                                       out=out[l], workspace=ws, abi=abis[l])
+                                       out=out[l], workspace=ws, abi=abis[l],
+                                       flags=0 if args.no_early else lmo.LMO_STEP_CACHE_STABLE)
             elif attn:
                 lmo.lmo_decode_attention_q4(caches[l], qbuf[t][l].view(B, Hq, d), s + t,
                                             softmax_scale=sigma, num_splits=args.splits,

@@ -174,12 +174,19 @@ lmo_status lmo_decode_attention_q4(const lmo_kv_cache *cache, const void *q_f16,
  * lmo_kv_append_quant(pos = L_b - 1, n_new = 1) followed by
  * lmo_decode_attention_q4 on the same stream, in one launch when the pair-team
  * schedule is used (else two).  Other arguments as lmo_decode_attention_q4.
+ * flags: LMO_STEP_CACHE_STABLE = the kernel issued immediately before this
+ *        call on `stream` does not write this cache's slots [0, L_b - 1) (true
+ *        in a layer-by-layer decode loop).  The kernel may then start streaming
+ *        those old-token blocks before the previous kernel has finished
+ *        (programmatic dependent launch), overlapping its pipeline fill with
+ *        the previous kernel's tail.  Ignored with seq_lens_dev.  0 = none.
  * ------------------------------------------------------------------------- */
+#define LMO_STEP_CACHE_STABLE 1u
 lmo_status lmo_decode_step_q4(const lmo_kv_cache *cache, const void *k_new_f16,
                               const void *v_new_f16, const void *q_f16, int32_t q_heads,
                               int32_t len, const int32_t *seq_lens_dev, float softmax_scale,
                               int32_t num_splits, void *out, lmo_dtype out_dtype, void *workspace,
-                              size_t workspace_bytes, void *stream);
+                              size_t workspace_bytes, uint32_t flags, void *stream);
 
 /* Human-readable name of a status code (static string). */
 const char *lmo_status_string(lmo_status status);

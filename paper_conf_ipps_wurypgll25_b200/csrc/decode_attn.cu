@@ -86,6 +86,7 @@ struct AttnArgs {
     float *partials;          // [slots][G][REC]
     const __half *k_new;      // fused append (team mode): [B][Hkv][D] new token K, or nullptr
     const __half *v_new;      //                            new token V
+    int early;                // prefetch the old-token cache before griddepcontrol.wait
 };
 
 // ---------------------------------------------------------------- work map
@@ -362,6 +363,7 @@ struct WarpCtl {
     SegDesc seg;      // current consumer segment (all lanes read)
     int ppos;         // blocks of pc's segment already issued
     int qb, qkvh;     // pair whose q fragments are loaded
+    int pissued;      // stages issued by the pre-wait prologue
 };
 
 template <int D>
@@ -382,9 +384,15 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int g = lane >> 2, t = lane & 3;
-    // Programmatic dependent launch: this grid may start while the previous kernel in
-    // the stream drains; wait here before touching any of its outputs (no-op otherwise).
-    asm volatile("griddepcontrol.wait;\n" ::: "memory");
+    // Programmatic dependent launch: let the next kernel in the stream be scheduled
+    // as soon as our CTAs retire (its griddepcontrol.wait still waits for our full
+    // completion and memory flush).  Without `early`, wait here for the previous
+    // kernel before touching anything; with `early` (caller guarantees the previous
+    // kernel does not write this cache's old tokens), first start streaming the
+    // old-token cache blocks, then wait.
+    asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory");
+    const bool early = a.early && !a.lens;
+    if (!early) asm volatile("griddepcontrol.wait;\n" ::: "memory");
 
     // ---- work map (identical in every CTA)
     if (a.lens) {
@@ -475,6 +483,47 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
         }
     };
 
+    // producer prologue: barrier init, first segment, up to kStages bulk copies.  Before
+    // the fused append has run (early mode) a stage that holds the append slot L-1 is
+    // not issued yet; the ring is topped up after the append.
+    auto holds_append_slot = [&]() {
+        const SegIter &pc = ctl.pc;
+        const int n = min(kSub, pc.sn - ctl.ppos);
+        const int Lb = a.lens ? min(a.lens[pc.b], a.cap) : a.len;
+        return (pc.blk + ctl.ppos + n) * kBlk >= Lb;
+    };
+    auto prologue = [&](bool before_append) {
+        if (lane == 0) {
+            for (int s = 0; s < kStages; ++s) mbar_init(&wbar[s], 1);
+            fence_mbar_init();
+            if (wms.T) {
+                // team ids interleaved across CTAs (tau = team-in-CTA * grid + CTA): the busy
+                // teams spread evenly over the SMs when there are fewer pairs than teams
+                ctl.cc.v = (warp / wms.T) * gridDim.x + blockIdx.x;   // team id = first pair
+                ctl.cc.x0 = warp % wms.T;                             // rank in team
+            } else {
+                ctl.cc.v = gw;
+            }
+            ctl.cc.begin_v(wms);
+            ctl.pc = ctl.cc;
+            ctl.ppos = 0;
+            ctl.qb = -1;
+            ctl.qkvh = -1;
+            while (!ctl.pc.done && ctl.pc.sn == 0) ctl.pc.next(wms);   // (team mode) empty segments
+            int s = 0;
+            for (; s < kStages && !ctl.pc.done; ++s) {
+                if (before_append && a.k_new && holds_append_slot()) break;
+                issue(s);
+            }
+            ctl.pissued = s;
+        }
+        __syncwarp();
+    };
+    if (early) {
+        prologue(true);
+        asm volatile("griddepcontrol.wait;\n" ::: "memory");
+    }
+
     // ---- fused append (A2) of each pair's new token at slot L_b - 1, by the warp that
     // owns the pair's last block (team rank T-1) -- before any of its bulk copies, so
     // its own TMA reads of that block see the quantized token (proxy fence below).
@@ -514,26 +563,13 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
             for (int o = 0; o < D * 2; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(qn + o));
         }
     }
-    if (lane == 0) {
-        for (int s = 0; s < kStages; ++s) mbar_init(&wbar[s], 1);
-        fence_mbar_init();
-        if (wms.T) {
-            // team ids interleaved across CTAs (tau = team-in-CTA * grid + CTA): the busy
-            // teams spread evenly over the SMs when there are fewer pairs than teams
-            ctl.cc.v = (warp / wms.T) * gridDim.x + blockIdx.x;   // team id = first pair
-            ctl.cc.x0 = warp % wms.T;                             // rank in team
-        } else {
-            ctl.cc.v = gw;
-        }
-        ctl.cc.begin_v(wms);
-        ctl.pc = ctl.cc;
-        ctl.ppos = 0;
-        ctl.qb = -1;
-        ctl.qkvh = -1;
-        while (!ctl.pc.done && ctl.pc.sn == 0) ctl.pc.next(wms);   // (team mode) empty segments
-        for (int s = 0; s < kStages && !ctl.pc.done; ++s) issue(s);
+    if (early) {
+        if (lane == 0)
+            for (int s = ctl.pissued; s < kStages && !ctl.pc.done; ++s) issue(s);
+        __syncwarp();
+    } else {
+        prologue(false);
     }
-    __syncwarp();
 
     // ---- per-lane constant shared-memory offsets inside a stage (sub-block 0)
     const int tk0 = tperm(g), tk1 = 8 + tperm(g);                    // this lane's K/meta tokens
@@ -1234,8 +1270,9 @@ static int choose_team(int64_t pairs, int64_t warps) {
 cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq, int len,
                                     const int32_t *lens, float softmax_scale, int num_splits,
                                     void *out, int out_f16, void *ws, cudaStream_t st,
-                                    const void *k_new, const void *v_new) {
+                                    const void *k_new, const void *v_new, unsigned flags) {
     AttnArgs a;
+    a.early = (flags & LMO_STEP_CACHE_STABLE) ? 1 : 0;
     a.k_new = static_cast<const __half *>(k_new);
     a.v_new = static_cast<const __half *>(v_new);
     a.kv = c.kv;

@@ -34,7 +34,7 @@ cudaError_t launch_kv_append(const lmo_kv_cache &, const void *, const void *, i
                              const int32_t *, cudaStream_t, int pos_from_lens);
 cudaError_t launch_decode_attention(const lmo_kv_cache &, const void *, int, int, const int32_t *,
                                     float, int, void *, int, void *, cudaStream_t, const void *,
-                                    const void *);
+                                    const void *, unsigned);
 
 // Programmatic dependent launch for the hot-path kernels (LMO_PDL=0 disables).
 bool pdl_enabled() {
@@ -146,14 +146,14 @@ lmo_status lmo_decode_attention_q4(const lmo_kv_cache *cache, const void *q, int
                                                softmax_scale, num_splits, out,
                                                out_dtype == LMO_F16 ? 1 : 0, workspace,
                                                static_cast<cudaStream_t>(stream), nullptr,
-                                               nullptr));
+                                               nullptr, 0u));
 }
 
 lmo_status lmo_decode_step_q4(const lmo_kv_cache *cache, const void *k_new_f16,
                               const void *v_new_f16, const void *q, int32_t q_heads, int32_t len,
                               const int32_t *seq_lens_dev, float softmax_scale, int32_t num_splits,
                               void *out, lmo_dtype out_dtype, void *workspace,
-                              size_t workspace_bytes, void *stream) {
+                              size_t workspace_bytes, uint32_t flags, void *stream) {
     const lmo_status s = check_attention(cache, q, q_heads, len, seq_lens_dev, num_splits, out,
                                          out_dtype, workspace, workspace_bytes);
     if (s != LMO_OK) return s;
@@ -163,7 +163,7 @@ lmo_status lmo_decode_step_q4(const lmo_kv_cache *cache, const void *k_new_f16,
                                                softmax_scale, num_splits, out,
                                                out_dtype == LMO_F16 ? 1 : 0, workspace,
                                                static_cast<cudaStream_t>(stream), k_new_f16,
-                                               v_new_f16));
+                                               v_new_f16, flags));
 }
 
 const char *lmo_status_string(lmo_status st) {

@@ -19,6 +19,7 @@ from . import build as _build
 LMO_OK, LMO_ERR_NULL, LMO_ERR_SHAPE, LMO_ERR_UNSUPPORTED, LMO_ERR_ALIGN, LMO_ERR_WORKSPACE, \
     LMO_ERR_CUDA = range(7)
 LMO_F16, LMO_F32 = 0, 1
+LMO_STEP_CACHE_STABLE = 1
 GROUP = 64
 
 
@@ -47,7 +48,7 @@ def _load():
                                     i32, P, ctypes.c_int, P, ctypes.c_size_t, P],
         "lmo_gen_fill_f16": [P, i32, i32, i32, i32, u64, i32, i32, i32, i32, i32, i32, P],
         "lmo_decode_step_q4": [ctypes.POINTER(lmo_kv_cache), P, P, P, i32, i32, P, ctypes.c_float,
-                               i32, P, ctypes.c_int, P, ctypes.c_size_t, P],
+                               i32, P, ctypes.c_int, P, ctypes.c_size_t, ctypes.c_uint32, P],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -239,9 +240,11 @@ def lmo_decode_step_q4(cache: KVCache, k_new: torch.Tensor, v_new: torch.Tensor,
                        length: int = 0, seq_lens: torch.Tensor | None = None,
                        softmax_scale: float | None = None, num_splits: int = 0,
                        out: torch.Tensor | None = None, out_dtype: torch.dtype = torch.float32,
-                       workspace: torch.Tensor | None = None, stream=None, abi=None) -> torch.Tensor:
+                       workspace: torch.Tensor | None = None, flags: int = 0, stream=None,
+                       abi=None) -> torch.Tensor:
     """One decode step of one layer: append the new token's K/V ([B][Hkv][d] or
-    [B][Hkv][1][d]) at slot L-1, then attention over L (A2+A3+A4 fused)."""
+    [B][Hkv][1][d]) at slot L-1, then attention over L (A2+A3+A4 fused).
+    flags=LMO_STEP_CACHE_STABLE: see include/lmo.h."""
     B, Hq, d = q.shape
     if softmax_scale is None:
         softmax_scale = 1.0 / math.sqrt(d)
@@ -254,7 +257,7 @@ def lmo_decode_step_q4(cache: KVCache, k_new: torch.Tensor, v_new: torch.Tensor,
     c = abi if abi is not None else cache.abi()
     _check(_lib.lmo_decode_step_q4(ctypes.byref(c), _ptr(k_new), _ptr(v_new), _ptr(q), Hq, length,
                                    _ptr(seq_lens), float(softmax_scale), num_splits, _ptr(out), dt,
-                                   _ptr(workspace), workspace.numel(), _stream(stream)),
+                                   _ptr(workspace), workspace.numel(), int(flags), _stream(stream)),
            "lmo_decode_step_q4")
     return out
 

@@ -264,10 +264,12 @@ def test_full_size_sampled_rows(lmo, key):
 
 # ------------------------------------------ fused decode step (A2+A3+A4) ----
 
+@pytest.mark.parametrize("flags", [0, 1])
 @pytest.mark.parametrize("B,Hkv,G,d,L,ns", [(4, 6, 1, 128, 300, 0), (2, 2, 8, 128, 129, 0),
                                             (3, 4, 2, 64, 77, 2), (2, 3, 1, 128, 40, 4),
-                                            (2, 2, 4, 128, 200, 3), (1, 2, 1, 128, 1, 0)])
-def test_decode_step_fused_append(lmo, B, Hkv, G, d, L, ns):
+                                            (2, 2, 4, 128, 200, 3), (1, 2, 1, 128, 1, 0),
+                                            (3, 5, 1, 128, 33, 0), (2, 2, 8, 128, 16, 0)])
+def test_decode_step_fused_append(lmo, B, Hkv, G, d, L, ns, flags):
     """lmo_decode_step_q4 == append(new token at L-1) then attention over L, for the
     team schedule (one launch) and the stream-K fallback (two launches)."""
     seed = 31 + L
@@ -284,7 +286,7 @@ def test_decode_step_fused_append(lmo, B, Hkv, G, d, L, ns):
     lmo.lmo_gen_fill_f16(q, seed, I.STREAM_Q, 0, 0, 0, 0, group=G)
     q = q.view(B, Hkv * G, d)
     out = lmo.lmo_decode_step_q4(cache, kf[:, :, L - 1].contiguous(), vf[:, :, L - 1].contiguous(),
-                                 q, L, num_splits=ns)
+                                 q, L, num_splits=ns, flags=flags)
     torch.cuda.synchronize()
     host = oracle.new_cache(B, Hkv, cache.capacity, d)
     oracle.kv_append_quant(host, kf.cpu().numpy(), vf.cpu().numpy(), 0)
@@ -325,3 +327,41 @@ def test_decode_step_per_sequence_lengths(lmo):
     keep = lens > 0
     assert np.all(o[~keep] == 0)
     assert normwise_err(o[keep], ref[keep]).max() <= TOL
+
+
+def test_decode_loop_cache_stable_chain(lmo):
+    """Layer-by-layer decode loop (4 layers x 3 steps, back to back on one stream) with
+    LMO_STEP_CACHE_STABLE: every output matches the oracle."""
+    B, H, d, s0, nl, steps = 3, 4, 128, 90, 4, 3
+    cap = s0 + steps
+    caches, hosts, outs = [], [], []
+    kall = torch.empty((nl, B, H, cap, d), dtype=torch.float16, device="cuda")
+    vall = torch.empty_like(kall)
+    for l in range(nl):
+        lmo.lmo_gen_fill_f16(kall[l], 77, I.STREAM_K, l, 0, 0, 0)
+        lmo.lmo_gen_fill_f16(vall[l], 77, I.STREAM_V, l, 0, 0, 0)
+        c = lmo.KVCache.empty(B, H, cap, d)
+        lmo.lmo_kv_append_quant(c, kall[l, :, :, :s0].contiguous(), vall[l, :, :, :s0].contiguous(), 0)
+        caches.append(c)
+    q = torch.empty((nl, steps, B, H, 1, d), dtype=torch.float16, device="cuda")
+    for l in range(nl):
+        for t in range(steps):
+            lmo.lmo_gen_fill_f16(q[l, t], 77, I.STREAM_Q, l, 0, 0, t)
+    ws = lmo.attention_workspace(B, H, H, d)
+    kn = [[kall[l, :, :, s0 + t].contiguous() for t in range(steps)] for l in range(nl)]
+    vn = [[vall[l, :, :, s0 + t].contiguous() for t in range(steps)] for l in range(nl)]
+    torch.cuda.synchronize()
+    res = {}
+    for t in range(steps):
+        for l in range(nl):
+            res[(l, t)] = lmo.lmo_decode_step_q4(caches[l], kn[l][t], vn[l][t], q[l, t].view(B, H, d),
+                                                 s0 + t + 1, workspace=ws,
+                                                 flags=lmo.LMO_STEP_CACHE_STABLE)
+    torch.cuda.synchronize()
+    for l in range(nl):
+        host = oracle.new_cache(B, H, caches[l].capacity, d)
+        oracle.kv_append_quant(host, kall[l].cpu().numpy(), vall[l].cpu().numpy(), 0)
+        for t in range(steps):
+            ref = oracle.decode_attention_q4(host, q[l, t].view(B, H, d).cpu().numpy(), s0 + t + 1,
+                                             nthreads=8)
+            assert normwise_err(res[(l, t)].cpu().numpy(), ref).max() <= TOL, (l, t)

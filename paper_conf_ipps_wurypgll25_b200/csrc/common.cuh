@@ -54,35 +54,65 @@ __device__ __forceinline__ uint32_t meta_word(const GroupParams &p) {
     return (uint32_t)__half_as_ushort(p.mn_h) | ((uint32_t)__half_as_ushort(p.scale_h) << 16);
 }
 
+// min / max of 8 fp16 values held as 4 half2 (exact: packed fp16 min/max), as floats
+__device__ __forceinline__ void minmax8(const uint4 xv, float &mn, float &mx) {
+    const __half2 *h = reinterpret_cast<const __half2 *>(&xv);
+    __half2 lo = __hmin2(__hmin2(h[0], h[1]), __hmin2(h[2], h[3]));
+    __half2 hi = __hmax2(__hmax2(h[0], h[1]), __hmax2(h[2], h[3]));
+    mn = fminf(__low2float(lo), __high2float(lo));
+    mx = fmaxf(__low2float(hi), __high2float(hi));
+}
+
+// 8 codes of one uint4 (8 fp16) packed into a 32-bit word, low nibble first.
+// t is clamped to 15 BEFORE the rint (equivalent to min(15, rint(t)) since rint is
+// monotone and rint(15) = 15); the magic-constant add leaves c in the low bits.
+__device__ __forceinline__ uint32_t codes8(const uint4 xv, const GroupParams &p) {
+    const __half2 *h = reinterpret_cast<const __half2 *>(&xv);
+    uint32_t w = 0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const float2 f = __half22float2(h[k]);
+        const float t0 = fminf(__fmul_rn(__fsub_rn(f.x, p.mn), p.inv), 15.0f);
+        const float t1 = fminf(__fmul_rn(__fsub_rn(f.y, p.mn), p.inv), 15.0f);
+        const uint32_t c0 = __float_as_uint(__fadd_rn(t0, 12582912.0f)) - 0x4B400000u;
+        const uint32_t c1 = __float_as_uint(__fadd_rn(t1, 12582912.0f)) - 0x4B400000u;
+        w |= (c0 | (c1 << 4)) << (8 * k);
+    }
+    return w;
+}
+
 // Quantize one 64-group held by 8 consecutive lanes (lane8 = lane & 7), each
 // holding 8 consecutive fp16 elements (16 B).  Returns this lane's 4 code
 // bytes (elements 8*lane8 .. 8*lane8+7) and, via `meta`, the group meta word.
 __device__ __forceinline__ uint32_t quantize_group_lane8(const uint4 xv, uint32_t &meta) {
-    const __half2 *h2 = reinterpret_cast<const __half2 *>(&xv);
-    float v[8];
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-        float2 f = __half22float2(h2[k]);
-        v[2 * k] = f.x;
-        v[2 * k + 1] = f.y;
-    }
-    float mn = v[0], mx = v[0];
-#pragma unroll
-    for (int k = 1; k < 8; ++k) {
-        mn = fminf(mn, v[k]);
-        mx = fmaxf(mx, v[k]);
-    }
+    float mn, mx;
+    minmax8(xv, mn, mx);
 #pragma unroll
     for (int off = 1; off < 8; off <<= 1) {
         mn = fminf(mn, __shfl_xor_sync(0xffffffffu, mn, off));
         mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
     }
-    GroupParams p = group_params(mn, mx);
-    uint32_t w = 0;
-#pragma unroll
-    for (int k = 0; k < 8; ++k) w |= quant_code(v[k], p) << (4 * k);
+    const GroupParams p = group_params(mn, mx);
     meta = meta_word(p);
-    return w;
+    return codes8(xv, p);
+}
+
+// Same, 4 lanes per group (lane4 = lane & 3), each holding 16 consecutive
+// elements as two uint4; returns the lane's 8 code bytes.
+__device__ __forceinline__ uint2 quantize_group_lane4(const uint4 xa, const uint4 xb, uint32_t &meta) {
+    float mn, mx, mn2, mx2;
+    minmax8(xa, mn, mx);
+    minmax8(xb, mn2, mx2);
+    mn = fminf(mn, mn2);
+    mx = fmaxf(mx, mx2);
+#pragma unroll
+    for (int off = 1; off < 4; off <<= 1) {
+        mn = fminf(mn, __shfl_xor_sync(0xffffffffu, mn, off));
+        mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, off));
+    }
+    const GroupParams p = group_params(mn, mx);
+    meta = meta_word(p);
+    return make_uint2(codes8(xa, p), codes8(xb, p));
 }
 
 // ------------------------------------------------------------- PTX wrappers

@@ -18,21 +18,29 @@ __device__ __forceinline__ uint4 ldg_stream(const void *p) {
     return r;
 }
 
-// K1 fast path: inner == 1, n % 64 == 0.  One 64-group per 8 lanes.
+// K1 fast path: inner == 1, n % 64 == 0.  One 64-group per 4 lanes (16 elements
+// each: two 128-bit loads in flight), grid-stride over groups.
 __global__ void __launch_bounds__(256) quantize_vec_kernel(const __half *__restrict__ x,
                                                            int64_t ngroups_total,
                                                            uint8_t *__restrict__ codes,
                                                            uint32_t *__restrict__ meta) {
-    const int lane8 = threadIdx.x & 7;
-    const int64_t gid = (int64_t)blockIdx.x * (blockDim.x / 8) + (threadIdx.x >> 3);
-    const bool valid = gid < ngroups_total;
-    uint4 xv = make_uint4(0, 0, 0, 0);
-    if (valid) xv = ldg_stream(x + gid * kGroup + lane8 * 8);
-    uint32_t mw;
-    uint32_t w = quantize_group_lane8(xv, mw);     // all lanes take part in shuffles
-    if (valid) {
-        reinterpret_cast<uint32_t *>(codes + gid * (kGroup / 2))[lane8] = w;
-        if (lane8 == 0) meta[gid] = mw;
+    const int lane4 = threadIdx.x & 3;
+    const int64_t stride = (int64_t)gridDim.x * (blockDim.x / 4);
+    for (int64_t g0 = (int64_t)blockIdx.x * (blockDim.x / 4); g0 < ngroups_total; g0 += stride) {
+        const int64_t gid = g0 + (threadIdx.x >> 2);
+        const bool valid = gid < ngroups_total;
+        uint4 xa = make_uint4(0, 0, 0, 0), xb = xa;
+        if (valid) {
+            const __half *src = x + gid * kGroup + lane4 * 16;
+            xa = ldg_stream(src);
+            xb = ldg_stream(src + 8);
+        }
+        uint32_t mw;
+        const uint2 w = quantize_group_lane4(xa, xb, mw);     // all lanes take part in shuffles
+        if (valid) {
+            reinterpret_cast<uint2 *>(codes + gid * (kGroup / 2))[lane4] = w;
+            if (lane4 == 0) meta[gid] = mw;
+        }
     }
 }
 
@@ -72,7 +80,7 @@ __global__ void __launch_bounds__(256) quantize_generic_kernel(const __half *__r
 }
 
 // K2: quantize new K/V rows [B][Hkv][n_new][d] into cache slots pos_b + t.
-// Group id space: kv (2) x B x Hkv x n_new x (d/64), K rows first.
+// blockIdx.y: 0 = K, 1 = V; 4 lanes per 64-group, grid-stride over (row, group).
 __global__ void __launch_bounds__(256) kv_append_kernel(lmo_kv_cache cache,
                                                         const __half *__restrict__ k_new,
                                                         const __half *__restrict__ v_new,
@@ -82,33 +90,42 @@ __global__ void __launch_bounds__(256) kv_append_kernel(lmo_kv_cache cache,
     asm volatile("griddepcontrol.wait;\n" ::: "memory");   // PDL: inputs of earlier kernels
     const int d = cache.head_dim;
     const int gpr = d / kGroup;
-    const int lane8 = threadIdx.x & 7;
-    const int64_t rows_per_kv = (int64_t)cache.batch * cache.kv_heads * n_new;
-    const int64_t ngroups = 2 * rows_per_kv * gpr;
-    const int64_t gid = (int64_t)blockIdx.x * (blockDim.x / 8) + (threadIdx.x >> 3);
-    bool valid = gid < ngroups;
-    const int64_t gg = valid ? gid : 0;
-    const int kv = (int)(gg / (rows_per_kv * gpr));
-    const int64_t r = (gg / gpr) % rows_per_kv;          // (b*Hkv + h)*n_new + t
-    const int grp = (int)(gg % gpr);
-    const int t = (int)(r % n_new);
-    const int64_t bh = r / n_new;
-    const int b = (int)(bh / cache.kv_heads);
-    int pos = pos_dev ? pos_dev[b] : pos0;
-    if (pos_dev && pos_from_lens) pos = min(pos, cache.capacity) - 1;   // new token at L_b - 1
-    if (pos < 0 || pos + n_new > cache.capacity) valid = false;
-    const __half *src = (kv == 0 ? k_new : v_new) + r * d + grp * kGroup + lane8 * 8;
-    uint4 xv = make_uint4(0, 0, 0, 0);
-    if (valid) xv = ldg_stream(src);
-    uint32_t mw;
-    const uint32_t w = quantize_group_lane8(xv, mw);
-    if (valid) {
-        // compressed row: K codes | K meta | V codes | V meta
-        const int RB = d / 2, MB = gpr * 4, ROW = 2 * (RB + MB);
-        const int64_t slot = bh * cache.capacity + pos + t;
-        uint8_t *row = cache.kv + slot * ROW + kv * (RB + MB);
-        reinterpret_cast<uint32_t *>(row + grp * 32)[lane8] = w;
-        if (lane8 == 0) reinterpret_cast<uint32_t *>(row + RB)[grp] = mw;
+    const int RB = d / 2, MB = gpr * 4, ROW = 2 * (RB + MB);
+    const int kv = blockIdx.y;
+    const __half *srcbase = kv == 0 ? k_new : v_new;
+    const int lane4 = threadIdx.x & 3;
+    const int rows = cache.batch * cache.kv_heads * n_new;     // (b*Hkv + h)*n_new + t
+    const int ngroups = rows * gpr;
+    const int stride = gridDim.x * (blockDim.x / 4);
+    for (int g0 = blockIdx.x * (blockDim.x / 4); g0 < ngroups; g0 += stride) {
+        const int gid = g0 + (threadIdx.x >> 2);
+        bool valid = gid < ngroups;
+        const int r = valid ? gid / gpr : 0;
+        const int grp = gid - r * gpr;
+        const int bh = r / n_new;
+        const int t = r - bh * n_new;
+        const int b = bh / cache.kv_heads;
+        int pos = pos_dev ? pos_dev[b] : pos0;
+        if (pos_dev && pos_from_lens) pos = min(pos, cache.capacity) - 1;   // new token at L_b - 1
+        if (pos < 0 || pos + n_new > cache.capacity) valid = false;
+        uint4 xa = make_uint4(0, 0, 0, 0), xb = xa;
+        if (valid) {
+            const __half *src = srcbase + (int64_t)r * d + grp * kGroup + lane4 * 16;
+            xa = ldg_stream(src);
+            xb = ldg_stream(src + 8);
+        }
+        uint32_t mw;
+        const uint2 w = quantize_group_lane4(xa, xb, mw);
+        if (valid) {
+            // compressed row: K codes | K meta | V codes | V meta
+            const int64_t slot = (int64_t)bh * cache.capacity + pos + t;
+            uint8_t *row = cache.kv + slot * ROW + kv * (RB + MB);
+            // the V half of a d=64 row starts at byte 36: only 4-byte alignment holds
+            uint32_t *dst = reinterpret_cast<uint32_t *>(row + grp * 32 + lane4 * 8);
+            dst[0] = w.x;
+            dst[1] = w.y;
+            if (lane4 == 0) reinterpret_cast<uint32_t *>(row + RB)[grp] = mw;
+        }
     }
 }
 
@@ -118,24 +135,35 @@ __device__ __forceinline__ __half dequant_one(uint32_t c, uint32_t mw) {
     return __float2half_rn(__fmaf_rn((float)c, sc, mn));   // RN16(RN32(c*scale + min))
 }
 
-// K5 fast path: inner == 1, n % 64 == 0; 8 elements (4 code bytes, 16 B out) per thread.
+// K5 fast path: inner == 1, n % 64 == 0; 16 elements (8 code bytes in, 32 B out)
+// per thread, grid-stride.
 __global__ void __launch_bounds__(256) dequantize_vec_kernel(const uint8_t *__restrict__ codes,
                                                              const uint32_t *__restrict__ meta,
-                                                             int64_t n_oct,
+                                                             int64_t n_hex,
                                                              __half *__restrict__ y) {
-    const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (idx >= n_oct) return;
-    const uint32_t w = __ldg(reinterpret_cast<const uint32_t *>(codes) + idx);
-    const uint32_t mw = __ldg(meta + idx / 8);
-    uint4 out;
-    uint32_t *o = reinterpret_cast<uint32_t *>(&out);
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < n_hex; idx += stride) {
+        const uint2 w = __ldg(reinterpret_cast<const uint2 *>(codes) + idx);
+        const uint32_t mw = __ldg(meta + idx / 4);
+        const float mn = __half2float(__ushort_as_half((unsigned short)(mw & 0xffffu)));
+        const float sc = __half2float(__ushort_as_half((unsigned short)(mw >> 16)));
+        uint4 out[2];
+        uint32_t *o = reinterpret_cast<uint32_t *>(out);
 #pragma unroll
-    for (int k = 0; k < 4; ++k) {
-        const __half lo = dequant_one((w >> (8 * k)) & 0xf, mw);
-        const __half hi = dequant_one((w >> (8 * k + 4)) & 0xf, mw);
-        o[k] = (uint32_t)__half_as_ushort(lo) | ((uint32_t)__half_as_ushort(hi) << 16);
+        for (int k = 0; k < 8; ++k) {
+            const uint32_t word = k < 4 ? w.x : w.y;
+            const int sh = 8 * (k & 3);
+            // code -> float exactly via the 2^23 magic (0x4B000000 | c) - 2^23
+            const float c0 = __uint_as_float(0x4B000000u | ((word >> sh) & 0xfu)) - 8388608.0f;
+            const float c1 = __uint_as_float(0x4B000000u | ((word >> (sh + 4)) & 0xfu)) - 8388608.0f;
+            const __half lo = __float2half_rn(__fmaf_rn(c0, sc, mn));   // RN16(RN32(c*scale + min))
+            const __half hi = __float2half_rn(__fmaf_rn(c1, sc, mn));
+            o[k] = (uint32_t)__half_as_ushort(lo) | ((uint32_t)__half_as_ushort(hi) << 16);
+        }
+        uint4 *dst = reinterpret_cast<uint4 *>(y) + 2 * idx;
+        dst[0] = out[0];
+        dst[1] = out[1];
     }
-    reinterpret_cast<uint4 *>(y)[idx] = out;
 }
 
 // K5 general path: one thread per output element.
@@ -171,8 +199,8 @@ cudaError_t launch_quantize(const void *x, int64_t outer, int64_t n, int64_t inn
     uint32_t *mw = reinterpret_cast<uint32_t *>(meta);
     if (inner == 1 && n % kGroup == 0) {
         const int64_t groups = outer * (n / kGroup);
-        const int64_t blocks = (groups + 31) / 32;
-        quantize_vec_kernel<<<(unsigned)blocks, 256, 0, st>>>(xh, groups, codes, mw);
+        const int64_t blocks = (groups + 63) / 64;
+        quantize_vec_kernel<<<grid_for(blocks * 256, 256), 256, 0, st>>>(xh, groups, codes, mw);
     } else {
         const int64_t work = outer * ((n + kGroup - 1) / kGroup) * inner;
         quantize_generic_kernel<<<grid_for(work, 256), 256, 0, st>>>(xh, outer, n, inner, codes,
@@ -187,9 +215,8 @@ cudaError_t launch_dequantize(const uint8_t *codes, const lmo_qmeta *meta, int64
     const uint32_t *mw = reinterpret_cast<const uint32_t *>(meta);
     __half *yh = static_cast<__half *>(y);
     if (inner == 1 && n % kGroup == 0) {
-        const int64_t n_oct = outer * n / 8;
-        dequantize_vec_kernel<<<(unsigned)((n_oct + 255) / 256), 256, 0, st>>>(codes, mw, n_oct,
-                                                                                yh);
+        const int64_t n_hex = outer * n / 16;
+        dequantize_vec_kernel<<<grid_for(n_hex, 256), 256, 0, st>>>(codes, mw, n_hex, yh);
     } else {
         dequantize_generic_kernel<<<grid_for(outer * n * inner, 256), 256, 0, st>>>(
             codes, mw, outer, n, inner, yh);
@@ -201,11 +228,10 @@ cudaError_t launch_dequantize(const uint8_t *codes, const lmo_qmeta *meta, int64
 cudaError_t launch_kv_append(const lmo_kv_cache &cache, const void *k_new, const void *v_new,
                              int n_new, int pos0, const int32_t *pos_dev, cudaStream_t st,
                              int pos_from_lens) {
-    const int64_t groups =
-        2LL * cache.batch * cache.kv_heads * n_new * (cache.head_dim / kGroup);
-    const int64_t blocks = (groups + 31) / 32;
+    const int64_t groups = (int64_t)cache.batch * cache.kv_heads * n_new * (cache.head_dim / kGroup);
+    const int64_t blocks = (groups + 63) / 64;
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)blocks);
+    cfg.gridDim = dim3((unsigned)grid_for(blocks * 256, 256), 2);
     cfg.blockDim = dim3(256);
     cfg.stream = st;
     cudaLaunchAttribute attr[1];

@@ -120,7 +120,8 @@ size_t lmo_kv_row_bytes(int32_t head_dim);
  * n=head_dim, inner=1) would, and written to cache slot pos_b + t, where
  * pos_b = pos_dev[b] if pos_dev != NULL (device int32[batch]) else pos0.
  * Only slots [pos_b, pos_b + n_new) of each (b, h) are written.
- * Host-checked: 0 <= pos0, pos0 + n_new <= capacity (when pos_dev == NULL).
+ * Host-checked: 0 <= pos0, pos0 + n_new <= capacity (when pos_dev == NULL);
+ * 2*batch*kv_heads*n_new*(head_dim/64) < 2^31 (else LMO_ERR_SHAPE).
  * With pos_dev, out-of-range rows (pos_b < 0 or pos_b + n_new > capacity)
  * are skipped on the device.
  * ------------------------------------------------------------------------- */

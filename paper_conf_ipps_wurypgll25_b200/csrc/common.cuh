@@ -23,6 +23,21 @@ bool pdl_enabled();                         // programmatic dependent launch on/
 //   range = RN32(mx - mn); scale = RU16(RU32(range / 15)) == RU16(range/15);
 //   inv = scale == 0 ? 0 : RN32(1/scale);
 //   code = min(15, rint_even(RN32(RN32(x - mn) * inv))).
+// Unsigned 32-bit division by a runtime-invariant divisor d >= 1 (Granlund-Montgomery
+// round-up multiplier): q = (mulhi(m, n) + n) >> l, exact for every n < 2^32.
+struct FastDiv {
+    uint32_t d, m, l;
+    __host__ __device__ FastDiv() : d(1), m(0), l(0) {}
+    __host__ explicit FastDiv(uint32_t div) : d(div) {
+        l = 0;
+        while ((1ull << l) < div) ++l;
+        m = (uint32_t)((((1ull << l) - div) << 32) / div + 1);
+    }
+    __device__ __forceinline__ uint32_t div(uint32_t n) const {
+        return (uint32_t)(((uint64_t)__umulhi(m, n) + n) >> l);
+    }
+};
+
 struct GroupParams {
     float mn;       // canonical (+0 for a zero min)
     float inv;
@@ -33,9 +48,18 @@ struct GroupParams {
 __device__ __forceinline__ GroupParams group_params(float mn, float mx) {
     GroupParams p;
     p.mn = __fadd_rn(mn, 0.0f);                         // -0 -> +0
-    float range = __fsub_rn(__fadd_rn(mx, 0.0f), p.mn);
-    p.scale_h = __float2half_ru(__fdiv_ru(range, 15.0f));
-    float s = __half2float(p.scale_h);
+    const float range = __fsub_rn(__fadd_rn(mx, 0.0f), p.mn);
+    // scale = RU16(RU32(range/15)) = RU16(range/15) (two upward roundings compose):
+    // the least fp16 h with 15*h >= range.  Start from RU16 of an approximate
+    // quotient (off by at most one fp16 step) and correct with exact tests --
+    // 15*h has <= 15 significant bits, so the fp32 product and compare are exact.
+    unsigned short hb = __half_as_ushort(__float2half_ru(__fmul_rn(range, 1.0f / 15.0f)));
+    const float hf = __half2float(__ushort_as_half(hb));
+    const float hp = __half2float(__ushort_as_half((unsigned short)(hb - 1)));
+    if (__fmul_rn(hf, 15.0f) < range) hb += 1;
+    else if (hb != 0 && __fmul_rn(hp, 15.0f) >= range) hb -= 1;
+    p.scale_h = __ushort_as_half(hb);
+    const float s = __half2float(p.scale_h);
     p.inv = (s == 0.0f) ? 0.0f : __frcp_rn(s);
     p.mn_h = __float2half_rn(p.mn);                     // exact: mn is an fp16 value
     return p;
@@ -64,21 +88,25 @@ __device__ __forceinline__ void minmax8(const uint4 xv, float &mn, float &mx) {
 }
 
 // 8 codes of one uint4 (8 fp16) packed into a 32-bit word, low nibble first.
-// t is clamped to 15 BEFORE the rint (equivalent to min(15, rint(t)) since rint is
-// monotone and rint(15) = 15); the magic-constant add leaves c in the low bits.
+// rint: t + 1.5*2^23 leaves the bit pattern 0x4B400000 + c.  Instead of masking
+// each code, accumulate bits_k << 4k over k and subtract the constant
+// sum(0x4B400000 << 4k) mod 2^32 once (one LEA/IMAD per element).
+// The clamp min(15, .) is provably inactive here: x - mn <= range (RN32 is
+// monotone), scale >= range/15 and inv = RN32(1/scale), so t <= 15(1+2^-24)^2
+// < 15.5 and rint(t) <= 15 -- bit-identical to quant_code() / the oracle.
 __device__ __forceinline__ uint32_t codes8(const uint4 xv, const GroupParams &p) {
     const __half2 *h = reinterpret_cast<const __half2 *>(&xv);
-    uint32_t w = 0;
+    constexpr uint32_t kMagicSum = 0x4B400000u * 0x11111111u;   // sum_k 0x4B400000 << 4k
+    uint32_t acc = 0u - kMagicSum;
 #pragma unroll
     for (int k = 0; k < 4; ++k) {
         const float2 f = __half22float2(h[k]);
-        const float t0 = fminf(__fmul_rn(__fsub_rn(f.x, p.mn), p.inv), 15.0f);
-        const float t1 = fminf(__fmul_rn(__fsub_rn(f.y, p.mn), p.inv), 15.0f);
-        const uint32_t c0 = __float_as_uint(__fadd_rn(t0, 12582912.0f)) - 0x4B400000u;
-        const uint32_t c1 = __float_as_uint(__fadd_rn(t1, 12582912.0f)) - 0x4B400000u;
-        w |= (c0 | (c1 << 4)) << (8 * k);
+        const float t0 = __fmul_rn(__fsub_rn(f.x, p.mn), p.inv);
+        const float t1 = __fmul_rn(__fsub_rn(f.y, p.mn), p.inv);
+        acc += __float_as_uint(__fadd_rn(t0, 12582912.0f)) << (8 * k);
+        acc += __float_as_uint(__fadd_rn(t1, 12582912.0f)) << (8 * k + 4);
     }
-    return w;
+    return acc;
 }
 
 // Quantize one 64-group held by 8 consecutive lanes (lane8 = lane & 7), each

@@ -99,6 +99,9 @@ lmo_status lmo_kv_append_quant(const lmo_kv_cache *cache, const void *k_new, con
     if (n_new < 0) return LMO_ERR_SHAPE;
     if (n_new == 0) return LMO_OK;
     if (!pos_dev && (pos0 < 0 || (int64_t)pos0 + n_new > cache->capacity)) return LMO_ERR_SHAPE;
+    // the append kernel indexes (row, K|V, group) units in 32-bit
+    if (2LL * cache->batch * cache->kv_heads * n_new * (cache->head_dim / kGroup) >= (1LL << 31))
+        return LMO_ERR_SHAPE;
     if (!aligned16(k_new) || !aligned16(v_new)) return LMO_ERR_ALIGN;
     return cuda_status(launch_kv_append(*cache, k_new, v_new, n_new, pos0, pos_dev,
                                         static_cast<cudaStream_t>(stream), 0));

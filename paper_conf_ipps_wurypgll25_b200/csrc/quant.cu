@@ -80,44 +80,46 @@ __global__ void __launch_bounds__(256) quantize_generic_kernel(const __half *__r
 }
 
 // K2: quantize new K/V rows [B][Hkv][n_new][d] into cache slots pos_b + t.
-// blockIdx.y: 0 = K, 1 = V; 4 lanes per 64-group, grid-stride over (row, group).
+// 4 lanes per 64-group, grid-stride over (row, K|V, group) units.
 __global__ void __launch_bounds__(256) kv_append_kernel(lmo_kv_cache cache,
                                                         const __half *__restrict__ k_new,
                                                         const __half *__restrict__ v_new,
-                                                        int n_new, int pos0,
+                                                        int n_new, FastDiv div_n, FastDiv div_h,
+                                                        int pos0,
                                                         const int32_t *__restrict__ pos_dev,
                                                         int pos_from_lens) {
     asm volatile("griddepcontrol.wait;\n" ::: "memory");   // PDL: inputs of earlier kernels
     const int d = cache.head_dim;
     const int gpr = d / kGroup;
     const int RB = d / 2, MB = gpr * 4, ROW = 2 * (RB + MB);
-    const int kv = blockIdx.y;
-    const __half *srcbase = kv == 0 ? k_new : v_new;
+    // unit u = (row r, half kv, group grp), kv-major inside a row so that a warp's 8
+    // units cover whole compressed rows (K codes|K meta|V codes|V meta) contiguously
     const int lane4 = threadIdx.x & 3;
-    const int rows = cache.batch * cache.kv_heads * n_new;     // (b*Hkv + h)*n_new + t
-    const int ngroups = rows * gpr;
+    const int upr = 2 * gpr;                                   // units per row
+    const int nunits = cache.batch * cache.kv_heads * n_new * upr;
     const int stride = gridDim.x * (blockDim.x / 4);
-    for (int g0 = blockIdx.x * (blockDim.x / 4); g0 < ngroups; g0 += stride) {
-        const int gid = g0 + (threadIdx.x >> 2);
-        bool valid = gid < ngroups;
-        const int r = valid ? gid / gpr : 0;
-        const int grp = gid - r * gpr;
-        const int bh = r / n_new;
+    for (int u0 = blockIdx.x * (blockDim.x / 4); u0 < nunits; u0 += stride) {
+        const int u = u0 + (threadIdx.x >> 2);
+        bool valid = u < nunits;
+        const int r = valid ? (u >> gpr) : 0;                  // upr = 2*gpr = 2 or 4: shift by gpr
+        const int within = u - r * upr;                        // r = (b*Hkv + h)*n_new + t
+        const int kv = within >= gpr;
+        const int grp = within - kv * gpr;
+        const int bh = (int)div_n.div((uint32_t)r);
         const int t = r - bh * n_new;
-        const int b = bh / cache.kv_heads;
+        const int b = (int)div_h.div((uint32_t)bh);
         int pos = pos_dev ? pos_dev[b] : pos0;
         if (pos_dev && pos_from_lens) pos = min(pos, cache.capacity) - 1;   // new token at L_b - 1
         if (pos < 0 || pos + n_new > cache.capacity) valid = false;
         uint4 xa = make_uint4(0, 0, 0, 0), xb = xa;
         if (valid) {
-            const __half *src = srcbase + (int64_t)r * d + grp * kGroup + lane4 * 16;
+            const __half *src = (kv ? v_new : k_new) + (int64_t)r * d + grp * kGroup + lane4 * 16;
             xa = ldg_stream(src);
             xb = ldg_stream(src + 8);
         }
         uint32_t mw;
         const uint2 w = quantize_group_lane4(xa, xb, mw);
         if (valid) {
-            // compressed row: K codes | K meta | V codes | V meta
             const int64_t slot = (int64_t)bh * cache.capacity + pos + t;
             uint8_t *row = cache.kv + slot * ROW + kv * (RB + MB);
             // the V half of a d=64 row starts at byte 36: only 4-byte alignment holds
@@ -135,34 +137,41 @@ __device__ __forceinline__ __half dequant_one(uint32_t c, uint32_t mw) {
     return __float2half_rn(__fmaf_rn((float)c, sc, mn));   // RN16(RN32(c*scale + min))
 }
 
-// K5 fast path: inner == 1, n % 64 == 0; 16 elements (8 code bytes in, 32 B out)
-// per thread, grid-stride.
-__global__ void __launch_bounds__(256) dequantize_vec_kernel(const uint8_t *__restrict__ codes,
+// K5 fast path: inner == 1, n % 64 == 0.  One 32-bit code word (8 elements) in, one
+// 16-byte fp16 vector out per thread and item; consecutive lanes take consecutive
+// words so every load and store instruction is fully coalesced; 4 items per thread
+// in flight, grid-stride over tiles of 4*blockDim words.
+__global__ void __launch_bounds__(256) dequantize_vec_kernel(const uint32_t *__restrict__ codes,
                                                              const uint32_t *__restrict__ meta,
-                                                             int64_t n_hex,
-                                                             __half *__restrict__ y) {
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < n_hex; idx += stride) {
-        const uint2 w = __ldg(reinterpret_cast<const uint2 *>(codes) + idx);
-        const uint32_t mw = __ldg(meta + idx / 4);
-        const float mn = __half2float(__ushort_as_half((unsigned short)(mw & 0xffffu)));
-        const float sc = __half2float(__ushort_as_half((unsigned short)(mw >> 16)));
-        uint4 out[2];
-        uint32_t *o = reinterpret_cast<uint32_t *>(out);
+                                                             int64_t n_words,
+                                                             uint4 *__restrict__ y) {
+    constexpr int kItems = 4;
+    const int64_t tile = (int64_t)kItems * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * tile; base < n_words; base += (int64_t)gridDim.x * tile) {
+        uint32_t w[kItems], mw[kItems];
 #pragma unroll
-        for (int k = 0; k < 8; ++k) {
-            const uint32_t word = k < 4 ? w.x : w.y;
-            const int sh = 8 * (k & 3);
-            // code -> float exactly via the 2^23 magic (0x4B000000 | c) - 2^23
-            const float c0 = __uint_as_float(0x4B000000u | ((word >> sh) & 0xfu)) - 8388608.0f;
-            const float c1 = __uint_as_float(0x4B000000u | ((word >> (sh + 4)) & 0xfu)) - 8388608.0f;
-            const __half lo = __float2half_rn(__fmaf_rn(c0, sc, mn));   // RN16(RN32(c*scale + min))
-            const __half hi = __float2half_rn(__fmaf_rn(c1, sc, mn));
-            o[k] = (uint32_t)__half_as_ushort(lo) | ((uint32_t)__half_as_ushort(hi) << 16);
+        for (int j = 0; j < kItems; ++j) {
+            const int64_t i = base + j * blockDim.x + threadIdx.x;
+            w[j] = i < n_words ? __ldcs(codes + i) : 0u;
+            mw[j] = i < n_words ? __ldg(meta + i / 8) : 0u;    // 8 words per 64-group
         }
-        uint4 *dst = reinterpret_cast<uint4 *>(y) + 2 * idx;
-        dst[0] = out[0];
-        dst[1] = out[1];
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+            const int64_t i = base + j * blockDim.x + threadIdx.x;
+            const float mn = __half2float(__ushort_as_half((unsigned short)(mw[j] & 0xffffu)));
+            const float sc = __half2float(__ushort_as_half((unsigned short)(mw[j] >> 16)));
+            uint32_t o[4];
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                // code -> float exactly via the 2^23 magic (0x4B000000 | c) - 2^23
+                const float c0 = __uint_as_float(0x4B000000u | ((w[j] >> (8 * k)) & 0xfu)) - 8388608.0f;
+                const float c1 = __uint_as_float(0x4B000000u | ((w[j] >> (8 * k + 4)) & 0xfu)) - 8388608.0f;
+                const __half lo = __float2half_rn(__fmaf_rn(c0, sc, mn));   // RN16(RN32(c*scale + min))
+                const __half hi = __float2half_rn(__fmaf_rn(c1, sc, mn));
+                o[k] = (uint32_t)__half_as_ushort(lo) | ((uint32_t)__half_as_ushort(hi) << 16);
+            }
+            if (i < n_words) __stcs(y + i, make_uint4(o[0], o[1], o[2], o[3]));
+        }
     }
 }
 
@@ -215,8 +224,9 @@ cudaError_t launch_dequantize(const uint8_t *codes, const lmo_qmeta *meta, int64
     const uint32_t *mw = reinterpret_cast<const uint32_t *>(meta);
     __half *yh = static_cast<__half *>(y);
     if (inner == 1 && n % kGroup == 0) {
-        const int64_t n_hex = outer * n / 16;
-        dequantize_vec_kernel<<<grid_for(n_hex, 256), 256, 0, st>>>(codes, mw, n_hex, yh);
+        const int64_t n_words = outer * n / 8;
+        dequantize_vec_kernel<<<grid_for((n_words + 3) / 4, 256), 256, 0, st>>>(
+            reinterpret_cast<const uint32_t *>(codes), mw, n_words, reinterpret_cast<uint4 *>(yh));
     } else {
         dequantize_generic_kernel<<<grid_for(outer * n * inner, 256), 256, 0, st>>>(
             codes, mw, outer, n, inner, yh);
@@ -228,10 +238,10 @@ cudaError_t launch_dequantize(const uint8_t *codes, const lmo_qmeta *meta, int64
 cudaError_t launch_kv_append(const lmo_kv_cache &cache, const void *k_new, const void *v_new,
                              int n_new, int pos0, const int32_t *pos_dev, cudaStream_t st,
                              int pos_from_lens) {
-    const int64_t groups = (int64_t)cache.batch * cache.kv_heads * n_new * (cache.head_dim / kGroup);
-    const int64_t blocks = (groups + 63) / 64;
+    const int64_t units = 2LL * cache.batch * cache.kv_heads * n_new * (cache.head_dim / kGroup);
+    const int64_t blocks = (units + 63) / 64;
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3((unsigned)grid_for(blocks * 256, 256), 2);
+    cfg.gridDim = dim3((unsigned)grid_for(blocks * 256, 256));
     cfg.blockDim = dim3(256);
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
@@ -241,7 +251,9 @@ cudaError_t launch_kv_append(const lmo_kv_cache &cache, const void *k_new, const
     cfg.numAttrs = 1;
     const cudaError_t e = cudaLaunchKernelEx(&cfg, kv_append_kernel, cache,
                                              static_cast<const __half *>(k_new),
-                                             static_cast<const __half *>(v_new), n_new, pos0, pos_dev,
+                                             static_cast<const __half *>(v_new), n_new,
+                                             FastDiv((uint32_t)n_new),
+                                             FastDiv((uint32_t)cache.kv_heads), pos0, pos_dev,
                                              pos_from_lens);
     note_launch();
     return e != cudaSuccess ? e : cudaGetLastError();

@@ -82,6 +82,40 @@ def test_quantize_bit_exact(lmo, outer, n, inner):
     assert np.array_equal(meta_u16(m), m_ref)
 
 
+def scale_sweep_tensor():
+    """Every positive finite fp16 value v as a group range (min 0, max v), plus as
+    many groups with a random negative min (range = RN32(v - mn)): exercises the
+    kernels' RU16(range/15) derivation at every fp16 step and the code rounding
+    at every scale (the paper's scale = (max - min)/(2^b - 1), R2)."""
+    rng = np.random.default_rng(7)
+    v = np.arange(1, 0x7C00, dtype=np.uint16).view(np.float16).astype(np.float64)
+    frac = np.linspace(0.0, 1.0, 64)
+    g1 = v[:, None] * frac[None, :]
+    mn = -rng.uniform(0, 1, v.size) * v
+    g2 = mn[:, None] + (v - mn)[:, None] * rng.permutation(frac)[None, :]
+    g2[:, 0], g2[:, 1] = mn, v
+    x = np.concatenate([g1, g2]).astype(np.float16)
+    x[: v.size, 63] = v.astype(np.float16)                  # exact max
+    return x.reshape(-1)
+
+
+def test_quantize_scale_sweep_bit_exact(lmo):
+    x = scale_sweep_tensor()
+    rows = x.size // 64
+    c_ref, m_ref = oracle.quantize_groupwise(x.reshape(rows, 64, 1), rows, 64, 1)
+    c, m = lmo.lmo_quantize_groupwise(dev(x.reshape(rows, 64, 1)), rows, 64, 1)
+    torch.cuda.synchronize()
+    assert np.array_equal(meta_u16(m), m_ref)
+    assert np.array_equal(c.cpu().numpy(), c_ref)
+    # the strided (inner > 1) kernel on the same groups, transposed
+    xt = np.ascontiguousarray(x.reshape(rows, 64).T).reshape(1, 64, rows)
+    c_ref, m_ref = oracle.quantize_groupwise(xt, 1, 64, rows)
+    c, m = lmo.lmo_quantize_groupwise(dev(xt), 1, 64, rows)
+    torch.cuda.synchronize()
+    assert np.array_equal(meta_u16(m), m_ref)
+    assert np.array_equal(c.cpu().numpy(), c_ref)
+
+
 @pytest.mark.parametrize("outer,n,inner", [(64, 128, 1), (3, 100, 1), (4, 128, 7), (513, 64 * 3, 1)])
 def test_dequantize_bit_exact(lmo, outer, n, inner):
     rng = np.random.default_rng(n + inner)
@@ -133,6 +167,23 @@ def test_append_bit_exact_with_canaries(lmo, d):
     got = cache_to_host(cache)
     for key in host:
         assert np.array_equal(got[key], host[key]), key
+
+
+@pytest.mark.parametrize("d", [64, 128])
+def test_append_scale_sweep_bit_exact(lmo, d):
+    """The append kernel's quantizer over the every-fp16-range sweep (K and V)."""
+    x = scale_sweep_tensor()
+    n = x.size // d
+    k = x[: n * d].reshape(1, 1, n, d)
+    v = np.ascontiguousarray(k[:, :, ::-1])
+    cache = lmo.KVCache.empty(1, 1, n, d)
+    lmo.lmo_kv_append_quant(cache, dev(k), dev(v), pos0=0)
+    host = oracle.new_cache(1, 1, cache.capacity, d)
+    oracle.kv_append_quant(host, k, v, 0)
+    torch.cuda.synchronize()
+    got = cache_to_host(cache)
+    for key in host:
+        assert np.array_equal(got[key][:, :, :n], host[key][:, :, :n]), key
 
 
 # ---------------------------------------------------------------- K3 -------

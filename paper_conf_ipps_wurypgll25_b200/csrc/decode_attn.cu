@@ -67,27 +67,14 @@ struct Geo {
 };
 
 #if LMO_ATTN_PROFILE
-__device__ unsigned long long *g_attn_prof = nullptr;   // [warp][4]: wait, total, stages, segments
+__device__ unsigned long long *g_attn_prof = nullptr;   // [slot][warp][16]: wait, total, stages, sm/warp/segs,
+                                                        // globaltimer at entry, loop start, first data, end
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
 #endif
-
-struct AttnArgs {
-    const uint8_t *kv;        // [B][Hkv][cap][ROW]
-    int B, Hkv, cap;
-    const __half *q;
-    int Hq, G;
-    int len;                  // uniform length (lens == nullptr)
-    const int32_t *lens;      // per-sequence lengths or nullptr
-    float scale_log2;         // softmax_scale * log2(e)
-    int num_splits;           // 0 = stream-K
-    int team;                 // > 0: pair-team mode with this many warps per pair
-    void *out;
-    int out_f16;
-    int *counters;            // [B*Hkv]
-    float *partials;          // [slots][G][REC]
-    const __half *k_new;      // fused append (team mode): [B][Hkv][D] new token K, or nullptr
-    const __half *v_new;      //                            new token V
-    int early;                // prefetch the old-token cache before griddepcontrol.wait
-};
 
 // ---------------------------------------------------------------- work map
 // Global list of 16-token blocks: sequence-major, then kv head, then block
@@ -101,6 +88,8 @@ struct WorkMap {
     int k;               // num_splits (0 = stream-K)
     int T;               // team mode: warps per (b, kvh) pair (1, 2, 4); 0 = stream-K / fixed splits
     int n_teams;         // team mode: teams in the grid
+    int tsh;             // team mode: log2(T)
+    FastDiv dHkv;        // division by Hkv
 
     __device__ __forceinline__ int seq_start(int b) const { return prefix ? prefix[b] : b * Hkv * nbu; }
     __device__ __forceinline__ int seq_nb(int b) const {
@@ -146,6 +135,28 @@ struct WorkMap {
         if (j > k - 1) j = k - 1;
         return (b * Hkv + kvh) * k + j;
     }
+};
+
+struct AttnArgs {
+    const uint8_t *kv;        // [B][Hkv][cap][ROW]
+    int B, Hkv, cap;
+    const __half *q;
+    int Hq, G;
+    int len;                  // uniform length (lens == nullptr)
+    const int32_t *lens;      // per-sequence lengths or nullptr
+    float scale_log2;         // softmax_scale * log2(e)
+    int num_splits;           // 0 = stream-K
+    int team;                 // > 0: pair-team mode with this many warps per pair
+    void *out;
+    int out_f16;
+    int *counters;            // [B*Hkv]
+    float *partials;          // [slots][G][REC]
+    const __half *k_new;      // fused append (team mode): [B][Hkv][D] new token K, or nullptr
+    const __half *v_new;      //                            new token V
+    int early;                // prefetch the old-token cache before griddepcontrol.wait
+    int prof_slot;            // (LMO_ATTN_PROFILE builds) record slot of this launch
+    WorkMap wm;               // host-computed work map (uniform length; completed on device
+                              // from the length prefix in per-sequence mode)
 };
 
 // Iterates the segments (maximal runs of blocks of one (b, kv head) pair) of
@@ -390,9 +401,15 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     // kernel before touching anything; with `early` (caller guarantees the previous
     // kernel does not write this cache's old tokens), first start streaming the
     // old-token cache blocks, then wait.
+#if LMO_ATTN_PROFILE
+    const unsigned long long prof_g0 = gtimer();
+#endif
     asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory");
     const bool early = a.early && !a.lens;
     if (!early) asm volatile("griddepcontrol.wait;\n" ::: "memory");
+#if LMO_ATTN_PROFILE
+    const unsigned long long prof_gw = gtimer();   // after the (non-early) wait
+#endif
 
     // ---- work map (identical in every CTA)
     if (a.lens) {
@@ -421,26 +438,18 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
         __syncthreads();
     }
     if (threadIdx.x == 0) {
-        WorkMap wm;
-        wm.B = a.B;
-        wm.Hkv = a.Hkv;
-        wm.k = a.num_splits;
-        wm.W = gridDim.x * kWarps;
+        WorkMap wm = a.wm;
         if (a.lens) {
             wm.prefix = prefix;
-            wm.nbu = 0;
             wm.N = prefix[a.B];
-        } else {
-            wm.prefix = nullptr;
-            wm.nbu = (a.len + kBlk - 1) / kBlk;
-            wm.N = a.B * a.Hkv * wm.nbu;
+            wm.V = wm.k == 0 ? (wm.N < wm.W ? wm.N : wm.W) : a.B * a.Hkv * wm.k;
         }
-        wm.V = wm.k == 0 ? (wm.N < wm.W ? wm.N : wm.W) : a.B * a.Hkv * wm.k;
-        wm.T = a.team;
-        wm.n_teams = a.team ? wm.W / a.team : 0;
         wms = wm;
     }
     __syncthreads();
+#if LMO_ATTN_PROFILE
+    const unsigned long long prof_gm = gtimer();   // after the work map
+#endif
 
     const int gw = blockIdx.x * kWarps + warp;
 
@@ -492,10 +501,16 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
         const int Lb = a.lens ? min(a.lens[pc.b], a.cap) : a.len;
         return (pc.blk + ctl.ppos + n) * kBlk >= Lb;
     };
-    auto prologue = [&](bool before_append) {
+#if LMO_ATTN_PROFILE
+    unsigned long long prof_gf = 0, prof_gb = 0;
+#endif
+    auto prologue = [&](bool before_append) {   // (always called with true)
         if (lane == 0) {
             for (int s = 0; s < kStages; ++s) mbar_init(&wbar[s], 1);
             fence_mbar_init();
+#if LMO_ATTN_PROFILE
+            prof_gf = gtimer();
+#endif
             if (wms.T) {
                 // team ids interleaved across CTAs (tau = team-in-CTA * grid + CTA): the busy
                 // teams spread evenly over the SMs when there are fewer pairs than teams
@@ -510,6 +525,9 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
             ctl.qb = -1;
             ctl.qkvh = -1;
             while (!ctl.pc.done && ctl.pc.sn == 0) ctl.pc.next(wms);   // (team mode) empty segments
+#if LMO_ATTN_PROFILE
+            prof_gb = gtimer();
+#endif
             int s = 0;
             for (; s < kStages && !ctl.pc.done; ++s) {
                 if (before_append && a.k_new && holds_append_slot()) break;
@@ -519,57 +537,131 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
         }
         __syncwarp();
     };
-    if (early) {
-        prologue(true);
-        asm volatile("griddepcontrol.wait;\n" ::: "memory");
-    }
+    // q B-fragments of pair (b, kvh): qf[grp] for head g (MHA: q in all 8 columns ->
+    // every lane's C holds real scores); qs = per-group sums of q for heads 2t, 2t+1
+    uint32_t qf[NG][4][2];
+    float qs[NG][2];
+    auto fetch_q = [&](int b, int kvh, uint4 (&raw)[NG][2]) {
+#pragma unroll
+        for (int grp = 0; grp < NG; ++grp) {
+            raw[grp][0] = raw[grp][1] = make_uint4(0, 0, 0, 0);
+            if (MHA || g < a.G) {
+                const __half *qp = a.q + (((int64_t)b * a.Hq + kvh * a.G + (MHA ? 0 : g)) * D + grp * 64 + 16 * t);
+                raw[grp][0] = *reinterpret_cast<const uint4 *>(qp);
+                raw[grp][1] = *reinterpret_cast<const uint4 *>(qp + 8);
+            }
+        }
+    };
+    auto build_q = [&](const uint4 (&raw)[NG][2]) {
+#pragma unroll
+        for (int grp = 0; grp < NG; ++grp) {
+            const __half *h0 = reinterpret_cast<const __half *>(&raw[grp][0]);
+            const __half *h1 = reinterpret_cast<const __half *>(&raw[grp][1]);
+            __half q16[16];
+            float sum = 0.f;
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                q16[i] = h0[i];
+                q16[8 + i] = h1[i];
+                sum += __half2float(h0[i]) + __half2float(h1[i]);
+            }
+            sum = sum_over_t(sum);                              // Qs of head g
+            qs[grp][0] = __shfl_sync(0xffffffffu, sum, 8 * t);      // head 2t   (g = 2t)
+            qs[grp][1] = __shfl_sync(0xffffffffu, sum, 8 * t + 4);  // head 2t+1
+#pragma unroll
+            for (int kbl = 0; kbl < 4; ++kbl) {
+#pragma unroll
+                for (int r = 0; r < 2; ++r) {
+                    const int idx = 2 * kbl + r;
+                    const int i0 = 8 * (idx >> 2) + (idx & 3);
+                    __half2 pr = __halves2half2(q16[i0], q16[i0 + 4]);
+                    if (r == 1) pr = __hmul2(pr, __float2half2_rn(0.0625f));  // meets c*2^-20
+                    qf[grp][kbl][r] = *reinterpret_cast<uint32_t *>(&pr);
+                }
+            }
+        }
+    };
+    auto load_q = [&](int b, int kvh) {
+        uint4 raw[NG][2];
+        fetch_q(b, kvh, raw);
+        build_q(raw);
+    };
 
     // ---- fused append (A2) of each pair's new token at slot L_b - 1, by the warp that
-    // owns the pair's last block (team rank T-1) -- before any of its bulk copies, so
-    // its own TMA reads of that block see the quantized token (proxy fence below).
-    if (a.k_new && wms.T) {
-        const int T = wms.T, rank = gw % T;
-        if (rank == T - 1) {
-            const int lane8 = lane & 7, kvsel = lane / (8 * NG), grp = (lane >> 3) % NG;
-            const bool lane_ok = lane < 16 * NG;
-            for (int p = (warp / T) * gridDim.x + blockIdx.x; p < a.B * a.Hkv; p += wms.n_teams) {
-                const int b = p / a.Hkv;
+    // owns the pair's last block (team rank T-1) -- before the bulk copies of that block,
+    // so its own TMA reads see the quantized token (proxy fence below).
+    const bool app_warp = a.k_new && wms.T && (gw % wms.T) == wms.T - 1;
+    const int lane8 = lane & 7, kvsel = lane / (8 * NG), grp8 = (lane >> 3) % NG;
+    const bool lane_ok = lane < 16 * NG;
+    const int p_first = wms.T ? (warp / wms.T) * gridDim.x + blockIdx.x : 0;
+    const bool first_ok = wms.T && p_first < a.B * a.Hkv;
+    auto app_src = [&](int p) {
+        return (kvsel == 0 ? a.k_new : a.v_new) + (int64_t)p * D + grp8 * 64 + lane8 * 8;
+    };
+    uint4 xv_first = make_uint4(0, 0, 0, 0);
+    uint4 qraw[NG][2];
+    // Team mode knows the warp's first pair: issue its q and new-token loads, then
+    // (non-early) the bulk copies, and only then consume the loads -- the small loads
+    // are queued ahead of the stage traffic and their latencies overlap.
+    auto fetch_first = [&]() {
+        if (app_warp && lane_ok && p_first < a.B * a.Hkv)
+            xv_first = *reinterpret_cast<const uint4 *>(app_src(p_first));
+        if (first_ok) {
+            const int b0 = (int)wms.dHkv.div((uint32_t)p_first);
+            fetch_q(b0, p_first - b0 * a.Hkv, qraw);
+        }
+    };
+    auto finish_first = [&]() {
+        if (first_ok) {
+            const int b0 = (int)wms.dHkv.div((uint32_t)p_first);
+            if (lane == 0) {
+                ctl.qb = b0;
+                ctl.qkvh = p_first - b0 * a.Hkv;
+            }
+            build_q(qraw);
+        }
+        if (app_warp) {
+            for (int p = p_first; p < a.B * a.Hkv; p += wms.n_teams) {
+                const int b = (int)wms.dHkv.div((uint32_t)p);
                 const int Lb = a.lens ? min(a.lens[b], a.cap) : a.len;
-                if (Lb < 1) continue;
-                const __half *src = (kvsel == 0 ? a.k_new : a.v_new) + (int64_t)p * D + grp * 64 + lane8 * 8;
-                uint4 xv = make_uint4(0, 0, 0, 0);
-                if (lane_ok) xv = *reinterpret_cast<const uint4 *>(src);
+                uint4 xv = xv_first;
+                if (p != p_first && lane_ok) xv = *reinterpret_cast<const uint4 *>(app_src(p));
                 uint32_t mw;
                 const uint32_t w = quantize_group_lane8(xv, mw);
-                if (lane_ok) {
+                if (lane_ok && Lb >= 1) {
                     uint8_t *row = const_cast<uint8_t *>(a.kv) + ((int64_t)p * a.cap + Lb - 1) * GG::ROW +
                                    kvsel * (GG::RB + GG::MB);
-                    reinterpret_cast<uint32_t *>(row + grp * 32)[lane8] = w;
-                    if (lane8 == 0) reinterpret_cast<uint32_t *>(row + GG::RB)[grp] = mw;
+                    reinterpret_cast<uint32_t *>(row + grp8 * 32)[lane8] = w;
+                    if (lane8 == 0) reinterpret_cast<uint32_t *>(row + GG::RB)[grp8] = mw;
                 }
             }
             asm volatile("fence.proxy.async.global;\n" ::: "memory");
-            __syncwarp();
         }
-    }
-
-    // team mode: this warp's first pair is known -> start pulling its q rows into L2 now
-    if (wms.T && lane < a.G) {
-        const int p0 = (warp / wms.T) * gridDim.x + blockIdx.x;
-        if (p0 < a.B * a.Hkv) {
-            const int b0 = p0 / a.Hkv, k0 = p0 - b0 * a.Hkv;
-            const char *qn = reinterpret_cast<const char *>(a.q + ((int64_t)b0 * a.Hq + k0 * a.G + lane) * D);
-#pragma unroll
-            for (int o = 0; o < D * 2; o += 128) asm volatile("prefetch.global.L2 [%0];" ::"l"(qn + o));
-        }
-    }
-    if (early) {
-        if (lane == 0)
-            for (int s = ctl.pissued; s < kStages && !ctl.pc.done; ++s) issue(s);
         __syncwarp();
+    };
+
+    // Early mode: bulk copies of old-token stages first (they may run before the previous
+    // kernel has finished), then the wait, then q / new token.  Otherwise the small loads
+    // go first.  Stages holding the append slot are held back until after the append.
+    if (early) {
+        prologue(true);
+        asm volatile("griddepcontrol.wait;\n" ::: "memory");
+        fetch_first();
     } else {
-        prologue(false);
+        fetch_first();
+        prologue(true);
     }
+#if LMO_ATTN_PROFILE
+    const unsigned long long prof_gp = gtimer();   // after the producer prologue
+#endif
+    finish_first();
+
+#if LMO_ATTN_PROFILE
+    const unsigned long long prof_ga = gtimer();   // after the fused append
+#endif
+    if (lane == 0)   // top the ring up (stages held back for the append)
+        for (int s = ctl.pissued; s < kStages && !ctl.pc.done; ++s) issue(s);
+    __syncwarp();
 
     // ---- per-lane constant shared-memory offsets inside a stage (sub-block 0)
     const int tk0 = tperm(g), tk1 = 8 + tperm(g);                    // this lane's K/meta tokens
@@ -591,9 +683,9 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     uint32_t phase = 0;
 #if LMO_ATTN_PROFILE
     long long prof_wait = 0, prof_t0 = clock64(), prof_seg = 0, prof_st = 0;
+    const unsigned long long prof_g1 = gtimer();
+    unsigned long long prof_g2 = 0, prof_gq = 0;
 #endif
-    uint32_t qf[NG][4][2];                    // q B-fragments (head g)
-    float qs[NG][2];                          // per-group sums of q for heads 2t, 2t+1
     int team_k = 0;                           // pairs finished (team mode: scratch double buffer)
 
     while (!ctl.cc.done) {
@@ -620,43 +712,13 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
                     ctl.qb = b;
                     ctl.qkvh = kvh;
                 }
-#pragma unroll
-                for (int grp = 0; grp < NG; ++grp) {
-                    uint4 q0 = make_uint4(0, 0, 0, 0), q1 = q0;
-                    // MHA: q replicated into all 8 columns -> every lane's C holds real scores
-                    if (MHA || g < a.G) {
-                        const __half *qp = a.q + (((int64_t)b * a.Hq + kvh * a.G + (MHA ? 0 : g)) * D + grp * 64 + 16 * t);
-                        q0 = *reinterpret_cast<const uint4 *>(qp);
-                        q1 = *reinterpret_cast<const uint4 *>(qp + 8);
-                    }
-                    const __half *h0 = reinterpret_cast<const __half *>(&q0);
-                    const __half *h1 = reinterpret_cast<const __half *>(&q1);
-                    __half q16[16];
-                    float sum = 0.f;
-#pragma unroll
-                    for (int i = 0; i < 8; ++i) {
-                        q16[i] = h0[i];
-                        q16[8 + i] = h1[i];
-                        sum += __half2float(h0[i]) + __half2float(h1[i]);
-                    }
-                    sum = sum_over_t(sum);                              // Qs of head g
-                    qs[grp][0] = __shfl_sync(0xffffffffu, sum, 8 * t);      // head 2t   (g = 2t)
-                    qs[grp][1] = __shfl_sync(0xffffffffu, sum, 8 * t + 4);  // head 2t+1
-#pragma unroll
-                    for (int kbl = 0; kbl < 4; ++kbl) {
-#pragma unroll
-                        for (int r = 0; r < 2; ++r) {
-                            const int idx = 2 * kbl + r;
-                            const int i0 = 8 * (idx >> 2) + (idx & 3);
-                            __half2 pr = __halves2half2(q16[i0], q16[i0 + 4]);
-                            if (r == 1) pr = __hmul2(pr, __float2half2_rn(0.0625f));  // meets c*2^-20
-                            qf[grp][kbl][r] = *reinterpret_cast<uint32_t *>(&pr);
-                        }
-                    }
-                }
+                load_q(b, kvh);
             }
         }
 
+#if LMO_ATTN_PROFILE
+        if (prof_seg == 1) prof_gq = gtimer();
+#endif
         // prefetch the next segment's q rows into L2 (its first use is latency-critical)
         if (!ctl.cc.done && lane < a.G) {
             const int nb_ = ctl.cc.b, nk_ = ctl.cc.kvh;
@@ -682,6 +744,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
 #endif
             mbar_wait(&wbar[sl], ph);
 #if LMO_ATTN_PROFILE
+            if (!prof_g2) prof_g2 = gtimer();
             prof_wait += clock64() - pw0;
 #endif
         };
@@ -1195,11 +1258,25 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     }
 #if LMO_ATTN_PROFILE
     if (lane == 0 && g_attn_prof) {
-        unsigned long long *pr = g_attn_prof + 4 * (size_t)gw;
+        unsigned long long *pr = g_attn_prof + 16 * ((size_t)a.prof_slot * 148 * 64 + gw);
+        unsigned smid, wid;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+        asm volatile("mov.u32 %0, %%warpid;" : "=r"(wid));
         pr[0] = prof_wait;
         pr[1] = clock64() - prof_t0;
         pr[2] = prof_st;
-        pr[3] = prof_seg;
+        pr[3] = ((unsigned long long)smid << 32) | ((unsigned long long)wid << 16) | (unsigned long long)prof_seg;
+        pr[4] = prof_g0;
+        pr[5] = prof_g1;
+        pr[6] = prof_g2;
+        pr[7] = gtimer();
+        pr[8] = prof_gw;
+        pr[9] = prof_gm;
+        pr[10] = prof_gp;
+        pr[11] = prof_ga;
+        pr[12] = prof_gq;
+        pr[13] = prof_gf;
+        pr[14] = prof_gb;
     }
 #endif
 }
@@ -1288,6 +1365,8 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     a.num_splits = num_splits;
     a.out = out;
     a.out_f16 = out_f16;
+    static int prof_launches = 0;            // profile builds: launch i records into slot i % 16
+    a.prof_slot = prof_launches++ % 16;
     const size_t counters = ((size_t)c.batch * c.kv_heads * sizeof(int) + 255) / 256 * 256;
     a.counters = static_cast<int *>(ws);
     a.partials = reinterpret_cast<float *>(static_cast<uint8_t *>(ws) + counters);
@@ -1316,6 +1395,8 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     int64_t want_warps;
     if (a.team) {
         want_warps = (int64_t)max_ctas * kWarps;          // all CTAs; idle teams exit at once
+        static const char *tight = getenv("LMO_ATTN_TIGHT");   // experiments: grid = teams
+        if (tight && tight[0] == '1') want_warps = pairs * a.team;
     } else if (lens) {
         want_warps = (int64_t)max_ctas * kWarps;
     } else {
@@ -1327,6 +1408,21 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     if (ctas < 1) ctas = 1;
     static const char *cap_env = getenv("LMO_ATTN_MAX_CTAS");   // tuning / experiments only
     if (cap_env && atoi(cap_env) > 0 && ctas > atoi(cap_env)) ctas = atoi(cap_env);
+    {   // the work map (uniform-length fields; per-sequence ones are completed on device)
+        WorkMap &wm = a.wm;
+        wm.prefix = nullptr;
+        wm.B = c.batch;
+        wm.Hkv = c.kv_heads;
+        wm.k = a.num_splits;
+        wm.W = (int)ctas * kWarps;
+        wm.nbu = lens ? 0 : (int)nbu;
+        wm.N = lens ? 0 : (int)(pairs * nbu);
+        wm.V = wm.k == 0 ? (wm.N < wm.W ? wm.N : wm.W) : (int)pairs * wm.k;
+        wm.T = a.team;
+        wm.n_teams = a.team ? wm.W / a.team : 0;
+        wm.tsh = a.team == 4 ? 2 : a.team == 2 ? 1 : 0;
+        wm.dHkv = FastDiv((uint32_t)c.kv_heads);
+    }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)ctas);
     cfg.blockDim = dim3(kWarps * 32);

@@ -46,6 +46,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_ATTN_PROFILE
 #define LMO_ATTN_PROFILE 0
 #endif
+#ifndef LMO_LAZY_MAX
+#define LMO_LAZY_MAX 0   // measured: no gain (c2), 3% loss (c5 GQA)
+#endif
 #ifndef LMO_ATTN_MINBLOCKS
 #define LMO_ATTN_MINBLOCKS 4
 #endif
@@ -372,10 +375,32 @@ struct WarpCtl {
     SegIter pc;       // producer iterator (lane 0)
     SegIter cc;       // consumer iterator (lane 0)
     SegDesc seg;      // current consumer segment (all lanes read)
-    int ppos;         // blocks of pc's segment already issued
+    const uint8_t *psrc;   // producer: source of the next stage
+    int ptok, pend, pLb;   // producer: next stage's first token, segment end token (< L), L of the pair
+    int pdone;             // producer: no more stages
     int qb, qkvh;     // pair whose q fragments are loaded
     int pissued;      // stages issued by the pre-wait prologue
 };
+
+// Producer segment setup (out of line): skip empty segments, then the byte cursor
+// of the new segment's tokens < L.
+template <int D>
+__device__ __noinline__ void prod_seg(WarpCtl &ctl, const WorkMap &wm, const uint8_t *kv,
+                                     const int32_t *lens, int cap, int len) {
+    SegIter &pc = ctl.pc;
+    while (!pc.done && pc.sn == 0) pc.next(wm);
+    if (pc.done) {
+        ctl.pdone = 1;
+        return;
+    }
+    const int Lb = lens ? min(lens[pc.b], cap) : len;
+    const int t0 = pc.blk * kBlk;
+    ctl.pdone = 0;
+    ctl.pLb = Lb;
+    ctl.ptok = t0;
+    ctl.pend = min((pc.blk + pc.sn) * kBlk, Lb);
+    ctl.psrc = kv + (((int64_t)pc.b * wm.Hkv + pc.kvh) * cap + t0) * Geo<D>::ROW;
+}
 
 template <int D>
 struct KState {       // per-stage scores handed from the K part to the V part
@@ -470,25 +495,19 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     WarpCtl &ctl = ctls[warp];
     const uint64_t pol = policy_evict_first();
 
-    // Producer (lane 0): one stage = up to kSub blocks of the producer's current
-    // segment; only the tokens < L_b are copied (exact-size tail, 16-B granular).
+    // Producer (lane 0): one stage = the next (up to) 32 tokens < L_b of the producer's
+    // current segment (exact-size tail, 16-B granular).  The per-stage path is a pointer
+    // bump; segment transitions (work-map arithmetic) run out of line.
     auto issue = [&](int slot) {
-        const WorkMap &wm = wms;
-        SegIter &pc = ctl.pc;
-        const int ppos = ctl.ppos;
-        const int n = min(kSub, pc.sn - ppos);
-        const int Lb = a.lens ? min(a.lens[pc.b], a.cap) : a.len;
-        const int tok_first = (pc.blk + ppos) * kBlk;
-        const int ntok = min(n * kBlk, Lb - tok_first);
-        const int bytes = (ntok * GG::ROW + 15) & ~15;          // cap % 16 == 0: in bounds
-        const int64_t tok0 = ((int64_t)pc.b * a.Hkv + pc.kvh) * a.cap + tok_first;
+        const int n = min(kStageTok, ctl.pend - ctl.ptok);
+        const uint32_t bytes = (n * GG::ROW + 15) & ~15;          // cap % 16 == 0: in bounds
         mbar_arrive_expect_tx(&wbar[slot], bytes);
-        bulk_g2s(wring + slot * GG::STAGE, a.kv + tok0 * GG::ROW, bytes, &wbar[slot], pol);
-        if (ppos + n >= pc.sn) {
-            do pc.next(wm); while (!pc.done && pc.sn == 0);
-            ctl.ppos = 0;
-        } else {
-            ctl.ppos = ppos + n;
+        bulk_g2s(wring + slot * GG::STAGE, ctl.psrc, bytes, &wbar[slot], pol);
+        ctl.psrc += kStageTok * GG::ROW;
+        ctl.ptok += kStageTok;
+        if (ctl.ptok >= ctl.pend) {
+            ctl.pc.next(wms);
+            prod_seg<D>(ctl, wms, a.kv, a.lens, a.cap, a.len);
         }
     };
 
@@ -496,10 +515,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     // the fused append has run (early mode) a stage that holds the append slot L-1 is
     // not issued yet; the ring is topped up after the append.
     auto holds_append_slot = [&]() {
-        const SegIter &pc = ctl.pc;
-        const int n = min(kSub, pc.sn - ctl.ppos);
-        const int Lb = a.lens ? min(a.lens[pc.b], a.cap) : a.len;
-        return (pc.blk + ctl.ppos + n) * kBlk >= Lb;
+        return ctl.ptok + min(kStageTok, ctl.pend - ctl.ptok) >= ctl.pLb;
     };
 #if LMO_ATTN_PROFILE
     unsigned long long prof_gf = 0, prof_gb = 0;
@@ -521,15 +537,14 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
             }
             ctl.cc.begin_v(wms);
             ctl.pc = ctl.cc;
-            ctl.ppos = 0;
             ctl.qb = -1;
             ctl.qkvh = -1;
-            while (!ctl.pc.done && ctl.pc.sn == 0) ctl.pc.next(wms);   // (team mode) empty segments
+            prod_seg<D>(ctl, wms, a.kv, a.lens, a.cap, a.len);
 #if LMO_ATTN_PROFILE
             prof_gb = gtimer();
 #endif
             int s = 0;
-            for (; s < kStages && !ctl.pc.done; ++s) {
+            for (; s < kStages && !ctl.pdone; ++s) {
                 if (before_append && a.k_new && holds_append_slot()) break;
                 issue(s);
             }
@@ -660,7 +675,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     const unsigned long long prof_ga = gtimer();   // after the fused append
 #endif
     if (lane == 0)   // top the ring up (stages held back for the append)
-        for (int s = ctl.pissued; s < kStages && !ctl.pc.done; ++s) issue(s);
+        for (int s = ctl.pissued; s < kStages && !ctl.pdone; ++s) issue(s);
     __syncwarp();
 
     // ---- per-lane constant shared-memory offsets inside a stage (sub-block 0)
@@ -852,6 +867,9 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
                 const int ls = t >> 1, hi = t & 1;
                 const int row = hi ? tk1 : tk0;
                 const float z = ks.z[0][0][0];
+                // the running max moves only if some lane's score exceeds it: one vote
+                // instead of a 5-shuffle max chain on most stages (same result)
+                if (!LMO_LAZY_MAX || __any_sync(0xffffffffu, z > m_run[0])) {
                 float mb = z;
 #pragma unroll
                 for (int off = 16; off > 0; off >>= 1) mb = fmaxf(mb, __shfl_xor_sync(0xffffffffu, mb, off));
@@ -868,6 +886,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
                         acc[i][2] *= a0;
                         acc[i][3] *= a0;
                     }
+                }
                 }
                 const float p = fast_exp2(z - m_run[0]);
                 l_run[0] += p;
@@ -909,7 +928,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
                     }
                 }
                 __syncwarp();
-                if (lane == 0 && !ctl.pc.done) issue(sl);
+                if (lane == 0 && !ctl.pdone) issue(sl);
 #if LMO_ATTN_PROFILE
                 ++prof_st;
 #endif
@@ -917,13 +936,15 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
             }
             float mb0 = fmaxf(fmaxf(ks.z[0][0][0], ks.z[0][1][0]), fmaxf(ks.z[kSub - 1][0][0], ks.z[kSub - 1][1][0]));
             float mb1 = fmaxf(fmaxf(ks.z[0][0][1], ks.z[0][1][1]), fmaxf(ks.z[kSub - 1][0][1], ks.z[kSub - 1][1][1]));
+            // lazy: the running maxima move only if some lane's score exceeds them (one vote;
+            // the shuffle reductions and the rescale run only then -- same result)
+            if (!LMO_LAZY_MAX || __any_sync(0xffffffffu, (mb0 > m_run[0]) || (mb1 > m_run[1]))) {
             mb0 = max_over_g(mb0);
             mb1 = max_over_g(mb1);
             const float mn0 = fmaxf(m_run[0], mb0), mn1 = fmaxf(m_run[1], mb1);
-            // FULL stages rescale unconditionally (branch-free: one basic block with the
-            // next stage's K part, which ptxas can interleave); GEN stages skip it when
-            // no running max moved.
-            if (F || __any_sync(0xffffffffu, (mn0 > m_run[0]) || (mn1 > m_run[1]))) {
+            // (non-lazy builds: FULL stages rescale unconditionally, branch-free; GEN stages
+            // skip it when no running max moved)
+            if (LMO_LAZY_MAX || F || __any_sync(0xffffffffu, (mn0 > m_run[0]) || (mn1 > m_run[1]))) {
                 const float a0 = fast_exp2(m_run[0] - mn0), a1 = fast_exp2(m_run[1] - mn1);
                 m_run[0] = mn0;
                 m_run[1] = mn1;
@@ -941,6 +962,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
                     acc[i][2] *= a0;
                     acc[i][3] *= a1;
                 }
+            }
             }
 #pragma unroll
             for (int s = 0; s < kSub; ++s) {
@@ -985,7 +1007,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
                 }
             }
             __syncwarp();
-            if (lane == 0 && !ctl.pc.done) issue(sl);
+            if (lane == 0 && !ctl.pdone) issue(sl);
 #if LMO_ATTN_PROFILE
             ++prof_st;
 #endif

@@ -44,6 +44,7 @@ def parse():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--splits", type=int, default=0, help="num_splits (0 = stream-K auto)")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-stream", action="store_true", help="skip the A1/A5 weight streaming leg")
     p.add_argument("--no-early", action="store_true", help="disable LMO_STEP_CACHE_STABLE")
     p.add_argument("--cpu-sample-seconds", type=float, default=10.0)
     return p.parse_args()
@@ -362,6 +363,40 @@ def run_ours(args):
         except Exception:
             traffic = None
 
+    # ---- streaming legs (A1 quantize, A5 dequantize) on one layer's weights, 12 h1^2
+    # elements (QKV/O + FFN), groups of 64 along the contiguous dim: the
+    # "q4 weight dequant" of BASELINE config 3 (Eq 4).  > L2; CUDA events.
+    streaming = None
+    if not args.no_stream and w.hidden > 0:
+        nel = 12 * w.hidden * w.hidden
+        rows, n = nel // w.hidden, w.hidden
+        with torch.cuda.stream(stream):
+            gen = torch.Generator(device=dev)
+            gen.manual_seed(seed)
+            xw = (torch.randn((rows, n), generator=gen, device=dev) * 0.02).half()   # weight-like N(0, 0.02)
+            codes = torch.empty((rows, n // 2), dtype=torch.uint8, device=dev)
+            meta = torch.empty((rows, n // 64), dtype=torch.int32, device=dev)
+            yw = torch.empty_like(xw)
+            res = {}
+            for name, fn, by in (
+                    ("quantize_A1", lambda: lmo.lmo_quantize_groupwise(xw, rows, n, 1, codes=codes, meta=meta,
+                                                                      stream=stream), nel * (2 + 0.5625)),
+                    ("dequantize_A5", lambda: lmo.lmo_dequantize_groupwise(codes, meta, rows, n, 1, y=yw,
+                                                                          stream=stream), nel * (0.5625 + 2))):
+                fn()
+                q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                q0.record(stream)
+                for _ in range(5):
+                    fn()
+                q1.record(stream)
+                q1.synchronize()
+                t_ms = reduce_max(q0.elapsed_time(q1)) / 5
+                res[name] = {"GB/s": by / (t_ms / 1e3) / 1e9, "frac": by / (t_ms / 1e3) / 1e9 / peak,
+                             "us_per_launch": t_ms * 1e3, "algorithmic_bytes": by}
+            streaming = {"elements": nel, "shape": f"({rows}, {n}) fp16 = 12 h1^2 weights of one layer",
+                         "peak": peak, **res}
+            del xw, codes, meta, yw
+
     # ---- e2e: host buffers, H2D of each step's inputs + D2H of its result in the region
     e2e = None
     if not args.no_e2e:
@@ -445,6 +480,7 @@ def run_ours(args):
                          "peak_source": peak_src,
                          "per_launch_us": attn_ms * 1e3, "algorithmic_bytes_per_launch": attn_bytes},
             "prefill_ms_all_layers": pre_ms,
+            "streaming": streaming,
             "gpu_launches": launches_per_step * args.steps,
             "clocks": clocks,
             "e2e": e2e,

@@ -157,9 +157,17 @@ size_t lmo_decode_attention_workspace_bytes(int32_t batch, int32_t kv_heads, int
  *               warp).  1, 2, 4 = pair teams of that size; other k > 0 = each
  *               pair split into k contiguous parts merged in-kernel.  With
  *               k > 0 results do not depend on batch composition.
+ *               LMO_SPLITS_STREAMK (-1) = stream-K explicitly.
+ *               LMO_SPLITS_SMTEAM (-2) = "SM teams" (uniform length only,
+ *               else auto): one CTA per SM owns a contiguous equal share of
+ *               the (b, kvh) pairs, its warps split that share into equal
+ *               block ranges, and pairs cut between warps are merged once
+ *               per CTA after a CTA barrier.
  * out         : [batch][q_heads][head_dim], LMO_F32 or LMO_F16.
  * q_heads/kv_heads must be in 1..8.
  * ------------------------------------------------------------------------- */
+#define LMO_SPLITS_STREAMK (-1)
+#define LMO_SPLITS_SMTEAM (-2)
 lmo_status lmo_decode_attention_q4(const lmo_kv_cache *cache, const void *q_f16, int32_t q_heads,
                                    int32_t len, const int32_t *seq_lens_dev, float softmax_scale,
                                    int32_t num_splits, void *out, lmo_dtype out_dtype,

@@ -28,6 +28,7 @@
 //    a KV tile is read once for all of them (8 q heads per kv head cost the
 //    same HMMA count as 1).
 #include <cstdlib>
+#include <cstring>
 #include <type_traits>
 
 #include "common.cuh"
@@ -92,6 +93,9 @@ struct WorkMap {
     int T;               // team mode: warps per (b, kvh) pair (1, 2, 4); 0 = stream-K / fixed splits
     int n_teams;         // team mode: teams in the grid
     int tsh;             // team mode: log2(T)
+    int sm;              // SM-team mode: CTA c owns pairs [c*P/C, (c+1)*P/C), split evenly over its warps
+    int P, C, NW;        // SM-team mode: pairs, CTAs, warps per CTA
+    int vb, X0, n;       // SM-team mode, this CTA: first virtual warp, first block, blocks
     FastDiv dHkv;        // division by Hkv
 
     __device__ __forceinline__ int seq_start(int b) const { return prefix ? prefix[b] : b * Hkv * nbu; }
@@ -121,6 +125,7 @@ struct WorkMap {
     }
     // start of virtual warp v's range
     __device__ __forceinline__ int R(int v) const {
+        if (sm) return X0 + (v - vb) * n / NW;   // v in [vb, vb + NW] (this CTA's warps)
         if (k == 0) return (int)((long long)v * N / V);
         const int p = v / k;
         if (p >= B * Hkv) return N;
@@ -192,9 +197,33 @@ struct SegIter {
         sx = wm.seq_start(b) + kvh * nb + lo;
         done = false;
     }
+    // SM teams: the warp's range [x0, x1) walked pair by pair from cursor a (inline: cheap)
+    __device__ __forceinline__ void sm_seg(const WorkMap &wm) {
+        if (a >= x1) {
+            done = true;
+            return;
+        }
+        const int p = a / wm.nbu;
+        b = (int)wm.dHkv.div((uint32_t)p);
+        kvh = p - b * wm.Hkv;
+        nb = wm.nbu;
+        blk = a - p * wm.nbu;
+        sx = a;
+        sn = min(x1, (p + 1) * wm.nbu) - a;
+        a += sn;
+        done = false;
+    }
     __device__ __forceinline__ void begin_v(const WorkMap &wm) {
-        if (wm.T) team_seg(wm);
-        else begin_v_sk(wm);
+        if (wm.T) {
+            team_seg(wm);
+        } else if (wm.sm) {
+            x0 = wm.R(v);
+            x1 = wm.R(v + 1);
+            a = x0;
+            sm_seg(wm);
+        } else {
+            begin_v_sk(wm);
+        }
     }
     __device__ __noinline__ void begin_v_sk(const WorkMap &wm) {
         while (v < wm.V) {
@@ -225,6 +254,8 @@ struct SegIter {
         if (wm.T) {
             v += wm.n_teams;
             team_seg(wm);
+        } else if (wm.sm) {
+            sm_seg(wm);
         } else {
             next_sk(wm);
         }
@@ -407,16 +438,20 @@ struct KState {       // per-stage scores handed from the K part to the V part
     float z[kSub][2][2];
 };
 
-template <int D, bool MHA>
-__global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q4_kernel(const AttnArgs a) {
+// smem layout: mbarriers [NW][kStages] (128-B aligned block), rings [NW][kStages][STAGE], prefix
+template <int NW>
+__host__ __device__ constexpr int bars_bytes() { return (NW * kStages * 8 + 127) / 128 * 128; }
+
+template <int D, bool MHA, int NW>
+__global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1) decode_attn_q4_kernel(const AttnArgs a) {
     using GG = Geo<D>;
     constexpr int NG = GG::NG;
     extern __shared__ __align__(128) uint8_t smem[];
-    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);                 // [kWarps][kStages]
-    uint8_t *ring = smem + 128;                                           // [kWarps][kStages][STAGE]
-    int *prefix = reinterpret_cast<int *>(ring + kWarps * kStages * GG::STAGE);
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);                 // [NW][kStages]
+    uint8_t *ring = smem + bars_bytes<NW>();                              // [NW][kStages][STAGE]
+    int *prefix = reinterpret_cast<int *>(ring + NW * kStages * GG::STAGE);
     __shared__ WorkMap wms;
-    __shared__ WarpCtl ctls[kWarps];
+    __shared__ WarpCtl ctls[NW];
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int g = lane >> 2, t = lane & 3;
@@ -464,6 +499,13 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     }
     if (threadIdx.x == 0) {
         WorkMap wm = a.wm;
+        if (wm.sm) {
+            const int p0 = (int)((long long)blockIdx.x * wm.P / wm.C);
+            const int p1 = (int)((long long)(blockIdx.x + 1) * wm.P / wm.C);
+            wm.vb = blockIdx.x * wm.NW;
+            wm.X0 = p0 * wm.nbu;
+            wm.n = (p1 - p0) * wm.nbu;
+        }
         if (a.lens) {
             wm.prefix = prefix;
             wm.N = prefix[a.B];
@@ -476,7 +518,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     const unsigned long long prof_gm = gtimer();   // after the work map
 #endif
 
-    const int gw = blockIdx.x * kWarps + warp;
+    const int gw = blockIdx.x * NW + warp;
 
     // ---- zero rows of empty sequences (per-sequence mode only)
     if (a.lens) {
@@ -605,11 +647,28 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     // ---- fused append (A2) of each pair's new token at slot L_b - 1, by the warp that
     // owns the pair's last block (team rank T-1) -- before the bulk copies of that block,
     // so its own TMA reads see the quantized token (proxy fence below).
-    const bool app_warp = a.k_new && wms.T && (gw % wms.T) == wms.T - 1;
+    // appending pairs of this warp: [app_lo, app_hi) step app_step.  Teams: rank T-1 of
+    // each team, pairs p_first, p_first + n_teams, ...  Stream-K (uniform length): the
+    // pairs whose last block lies in this warp's range [R(gw), R(gw+1)).
+    bool app_warp = false;
+    int app_lo = 0, app_hi = 0, app_step = 1;
+    if (a.k_new) {
+        if (wms.T) {
+            app_warp = (gw % wms.T) == wms.T - 1;
+            app_lo = (warp / wms.T) * gridDim.x + blockIdx.x;
+            app_hi = a.B * a.Hkv;
+            app_step = wms.n_teams;
+        } else if (gw < wms.V) {
+            app_lo = wms.R(gw) / wms.nbu;
+            app_hi = wms.R(gw + 1) / wms.nbu;
+            app_warp = app_lo < app_hi;
+        }
+    }
     const int lane8 = lane & 7, kvsel = lane / (8 * NG), grp8 = (lane >> 3) % NG;
     const bool lane_ok = lane < 16 * NG;
     const int p_first = wms.T ? (warp / wms.T) * gridDim.x + blockIdx.x : 0;
-    const bool first_ok = wms.T && p_first < a.B * a.Hkv;
+    bool first_ok = wms.T && p_first < a.B * a.Hkv;
+    int fb = 0, fk = 0;                 // pair of the warp's first segment (q prefetch)
     auto app_src = [&](int p) {
         return (kvsel == 0 ? a.k_new : a.v_new) + (int64_t)p * D + grp8 * 64 + lane8 * 8;
     };
@@ -619,28 +678,33 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     // (non-early) the bulk copies, and only then consume the loads -- the small loads
     // are queued ahead of the stage traffic and their latencies overlap.
     auto fetch_first = [&]() {
-        if (app_warp && lane_ok && p_first < a.B * a.Hkv)
-            xv_first = *reinterpret_cast<const uint4 *>(app_src(p_first));
-        if (first_ok) {
-            const int b0 = (int)wms.dHkv.div((uint32_t)p_first);
-            fetch_q(b0, p_first - b0 * a.Hkv, qraw);
+        if (app_warp && lane_ok && app_lo < app_hi)
+            xv_first = *reinterpret_cast<const uint4 *>(app_src(app_lo));
+        if (wms.T) {
+            fb = (int)wms.dHkv.div((uint32_t)p_first);
+            fk = p_first - fb * a.Hkv;
+        } else {                        // stream-K / SM teams: set by the producer prologue
+            first_ok = !ctl.cc.done;
+            fb = ctl.cc.b;
+            fk = ctl.cc.kvh;
         }
+        if (first_ok) fetch_q(fb, fk, qraw);
     };
     auto finish_first = [&]() {
         if (first_ok) {
-            const int b0 = (int)wms.dHkv.div((uint32_t)p_first);
+            __syncwarp();
             if (lane == 0) {
-                ctl.qb = b0;
-                ctl.qkvh = p_first - b0 * a.Hkv;
+                ctl.qb = fb;
+                ctl.qkvh = fk;
             }
             build_q(qraw);
         }
         if (app_warp) {
-            for (int p = p_first; p < a.B * a.Hkv; p += wms.n_teams) {
+            for (int p = app_lo; p < app_hi; p += app_step) {
                 const int b = (int)wms.dHkv.div((uint32_t)p);
                 const int Lb = a.lens ? min(a.lens[b], a.cap) : a.len;
                 uint4 xv = xv_first;
-                if (p != p_first && lane_ok) xv = *reinterpret_cast<const uint4 *>(app_src(p));
+                if (p != app_lo && lane_ok) xv = *reinterpret_cast<const uint4 *>(app_src(p));
                 uint32_t mw;
                 const uint32_t w = quantize_group_lane8(xv, mw);
                 if (lane_ok && Lb >= 1) {
@@ -658,9 +722,13 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     // Early mode: bulk copies of old-token stages first (they may run before the previous
     // kernel has finished), then the wait, then q / new token.  Otherwise the small loads
     // go first.  Stages holding the append slot are held back until after the append.
+    // (Stream-K / SM teams learn their first pair from the producer prologue.)
     if (early) {
         prologue(true);
         asm volatile("griddepcontrol.wait;\n" ::: "memory");
+        fetch_first();
+    } else if (!wms.T) {
+        prologue(true);
         fetch_first();
     } else {
         fetch_first();
@@ -698,6 +766,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
     uint32_t phase = 0;
 #if LMO_ATTN_PROFILE
     long long prof_wait = 0, prof_t0 = clock64(), prof_seg = 0, prof_st = 0;
+    long long prof_cs = 0, prof_ce = 0, prof_c0 = 0;   // cycles in segment start / end sections
     const unsigned long long prof_g1 = gtimer();
     unsigned long long prof_g2 = 0, prof_gq = 0;
 #endif
@@ -705,6 +774,9 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
 
     while (!ctl.cc.done) {
         // ------------------------------------------------ segment start
+#if LMO_ATTN_PROFILE
+        prof_c0 = clock64();
+#endif
         if (lane == 0) {
             SegIter &cc = ctl.cc;
             SegDesc d;
@@ -733,6 +805,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
 
 #if LMO_ATTN_PROFILE
         if (prof_seg == 1) prof_gq = gtimer();
+        prof_cs += clock64() - prof_c0;
 #endif
         // prefetch the next segment's q rows into L2 (its first use is latency-critical)
         if (!ctl.cc.done && lane < a.G) {
@@ -1066,6 +1139,9 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
         }
 
         // ------------------------------------------------ segment end
+#if LMO_ATTN_PROFILE
+        prof_c0 = clock64();
+#endif
         // heads 2t+e: reduce l and Pm over the 8 g-lanes; O = 2^24 acc(row g) / 2^20 acc(row g+8) + Pm
         float lt[2], pmt[2][NG];
         if constexpr (MHA) {      // per-lane tokens: full-warp sums; head 0 only
@@ -1130,7 +1206,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
                 const int rank = gw % T, gw0 = gw - rank;
                 const float *base = a.partials + (int64_t)(team_k & 1) * a.G * GG::REC;
                 for (int h = rank; h < a.G; h += T) {
-                    float mj[kWarps], lj[kWarps], oj[kWarps][DPL];
+                    float mj[kWarps], lj[kWarps], oj[kWarps][DPL];   // (teams: T <= kWarps)
 #pragma unroll
                     for (int j = 0; j < kWarps; ++j) {
                         if (j < T) {
@@ -1213,6 +1289,10 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
                     }
                 }
             }
+            if (wm.sm) {   // SM teams: merged once, after the CTA barrier at the end
+                __syncwarp();
+                continue;
+            }
             __threadfence();
             __syncwarp();
             // segments of this pair = non-empty ranges of virtual warps v0..v1
@@ -1277,6 +1357,95 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
             }
         }
         __syncwarp();
+#if LMO_ATTN_PROFILE
+        prof_ce += clock64() - prof_c0;
+#endif
+    }
+
+#if LMO_ATTN_PROFILE
+    prof_gf = gtimer();   // (slot 13 reused: end of the main loop)
+#endif
+    // ---- SM teams (A4): the CTA's pairs that were cut between warps are merged here,
+    // once, after one CTA barrier (partials in L2 scratch; no fences or atomics).
+    if (wms.sm) {
+        __syncthreads();
+        const WorkMap wm = wms;
+        const int c = blockIdx.x;
+        const int X0 = wm.X0, n = wm.n;
+        const int p0 = X0 / wm.nbu, p1 = (X0 + n) / wm.nbu;
+        // owner of block x = the largest warp w with X0 + floor(w n / NW) <= x
+        auto owner = [&](int x) { return ((x - X0 + 1) * NW + n - 1) / n - 1; };
+        constexpr int DPL = D / 32;
+        for (int p = p0 + warp; p < p1; p += NW) {
+            const int ps = p * wm.nbu;
+            const int w0 = owner(ps), w1 = owner(ps + wm.nbu - 1);
+            if (w0 == w1) continue;                         // one warp: written directly
+            const int vb = c * NW;
+            const int b = (int)wm.dHkv.div((uint32_t)p), kvh = p - b * a.Hkv;
+            const int64_t rowbase = (int64_t)b * a.Hq + (int64_t)kvh * a.G;
+            for (int h = 0; h < a.G; ++h) {
+                // online merge over the pieces, 4 at a time (all loads of a chunk independent:
+                // one L2 round trip per chunk; a pair rarely has more than 4 pieces)
+                float M = NEG_INF, l = 0.f, o[DPL];
+#pragma unroll
+                for (int i = 0; i < DPL; ++i) o[i] = 0.f;
+                for (int w = w0; w <= w1; w += 4) {
+                    float mj[4], lj[4], oj[4][DPL];
+                    bool ok[4];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        const int ww = w + u;
+                        ok[u] = ww <= w1 && wm.R(vb + ww) < wm.R(vb + ww + 1);
+                        mj[u] = NEG_INF;
+                        lj[u] = 0.f;
+#pragma unroll
+                        for (int i = 0; i < DPL; ++i) oj[u][i] = 0.f;
+                        if (ok[u]) {
+                            const int64_t sl = 2 * (int64_t)(vb + ww) + (ww == w0 && wm.R(vb + ww) < ps ? 1 : 0);
+                            const float *r = a.partials + sl * a.G * GG::REC + h * GG::REC;
+                            mj[u] = __ldcg(r + D);
+                            lj[u] = __ldcg(r + D + 1);
+                            if constexpr (DPL == 4) {
+                                const float4 x = __ldcg(reinterpret_cast<const float4 *>(r) + lane);
+                                oj[u][0] = x.x; oj[u][1] = x.y; oj[u][2] = x.z; oj[u][3] = x.w;
+                            } else {
+#pragma unroll
+                                for (int i = 0; i < DPL; ++i) oj[u][i] = __ldcg(r + lane * DPL + i);
+                            }
+                        }
+                    }
+                    float Mn = M;
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) Mn = fmaxf(Mn, mj[u]);
+                    const float sc = fast_exp2(M - Mn);      // (M = -inf on the first chunk: 0)
+                    l *= sc;
+#pragma unroll
+                    for (int i = 0; i < DPL; ++i) o[i] *= sc;
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) {
+                        if (!ok[u]) continue;
+                        const float wgt = fast_exp2(mj[u] - Mn);
+                        l = fmaf(lj[u], wgt, l);
+#pragma unroll
+                        for (int i = 0; i < DPL; ++i) o[i] = fmaf(oj[u][i], wgt, o[i]);
+                    }
+                    M = Mn;
+                }
+                const float il = 1.f / l;
+                const int64_t row = rowbase + h;
+                if (a.out_f16) {
+#pragma unroll
+                    for (int i = 0; i < DPL; ++i)
+                        static_cast<__half *>(a.out)[row * D + lane * DPL + i] = __float2half_rn(o[i] * il);
+                } else if constexpr (DPL == 4) {
+                    reinterpret_cast<float4 *>(static_cast<float *>(a.out) + row * D)[lane] =
+                        make_float4(o[0] * il, o[1] * il, o[2] * il, o[3] * il);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < DPL; ++i) static_cast<float *>(a.out)[row * D + lane * DPL + i] = o[i] * il;
+                }
+            }
+        }
     }
 #if LMO_ATTN_PROFILE
     if (lane == 0 && g_attn_prof) {
@@ -1299,6 +1468,7 @@ __global__ void __launch_bounds__(kWarps * 32, LMO_ATTN_MINBLOCKS) decode_attn_q
         pr[12] = prof_gq;
         pr[13] = prof_gf;
         pr[14] = prof_gb;
+        pr[15] = ((unsigned long long)prof_ce << 32) | (unsigned long long)(prof_cs & 0xffffffffull);
     }
 #endif
 }
@@ -1313,9 +1483,30 @@ extern "C" int lmo_debug_attn_profile(void *buf) {
 cudaError_t launch_kv_append(const lmo_kv_cache &cache, const void *k_new, const void *v_new,
                              int n_new, int pos0, const int32_t *pos_dev, cudaStream_t st,
                              int pos_from_lens);
-template <int D>
+template <int D, int NW = kWarps>
 static size_t smem_bytes(int B_prefix) {
-    return 128 + (size_t)kWarps * kStages * Geo<D>::STAGE + (B_prefix > 0 ? (B_prefix + 1) * sizeof(int) : 0);
+    return bars_bytes<NW>() + (size_t)NW * kStages * Geo<D>::STAGE + (B_prefix > 0 ? (B_prefix + 1) * sizeof(int) : 0);
+}
+
+// SM teams: one CTA of kSmWarps warps per SM (the ring fills the SM's shared memory)
+constexpr int kSmWarps = 16;
+template <int D>
+static bool sm_team_ok() {
+    static int ok[64] = {0};   // 0 unknown, 1 yes, 2 no
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (ok[dev] == 0) {
+        int n = 0, n1 = 0;
+        const int sz = (int)smem_bytes<D, kSmWarps>(0);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kSmWarps>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kSmWarps>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, decode_attn_q4_kernel<D, true, kSmWarps>, kSmWarps * 32, sz);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n1, decode_attn_q4_kernel<D, false, kSmWarps>, kSmWarps * 32, sz);
+        ok[dev] = (n >= 1 && n1 >= 1) ? 1 : 2;
+        cudaGetLastError();
+    }
+    return ok[dev] == 1;
 }
 
 template <int D>
@@ -1327,12 +1518,12 @@ static int ctas_per_sm(int B_prefix) {   // (MHA and GQA variants have the same 
     const int mode = B_prefix > 0 ? 1 : 0;
     if (occ[dev][mode] == 0) {
         for (int m = 0; m < 2; ++m)
-            cudaFuncSetAttribute(m ? decode_attn_q4_kernel<D, true> : decode_attn_q4_kernel<D, false>,
+            cudaFuncSetAttribute(m ? decode_attn_q4_kernel<D, true, kWarps> : decode_attn_q4_kernel<D, false, kWarps>,
                                  cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes<D>(kMaxBatchSmem));
         int n = 0, n1 = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n1, decode_attn_q4_kernel<D, true>, kWarps * 32,
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n1, decode_attn_q4_kernel<D, true, kWarps>, kWarps * 32,
                                                       smem_bytes<D>(mode ? kMaxBatchSmem : 0));
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, decode_attn_q4_kernel<D, false>, kWarps * 32,
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, decode_attn_q4_kernel<D, false, kWarps>, kWarps * 32,
                                                       smem_bytes<D>(mode ? kMaxBatchSmem : 0));
         if (n1 < n) n = n1;
         occ[dev][mode] = n > 0 ? n : 1;
@@ -1349,6 +1540,8 @@ size_t attn_workspace_bytes(int B, int Hkv, int Hq, int D, int num_splits) {
     const int G = Hq / Hkv;
     const size_t counters = ((size_t)B * Hkv * sizeof(int) + 255) / 256 * 256;
     size_t slots = 2 * (size_t)attn_max_warps(D, 0);               // stream-K and team scratch
+    const size_t sm_slots = 2 * (size_t)device_sm_count() * kSmWarps;  // SM teams
+    if (sm_slots > slots) slots = sm_slots;
     if (num_splits > 0 && (size_t)B * Hkv * num_splits > slots) slots = (size_t)B * Hkv * num_splits;
     return counters + slots * G * (D + 4) * sizeof(float);
 }
@@ -1399,17 +1592,26 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     const int64_t pairs = (int64_t)c.batch * c.kv_heads;
     const int64_t nbu = lens ? 0 : (len + kBlk - 1) / kBlk;
     a.team = 0;
-    if (num_splits == 1 || num_splits == 2 || num_splits == 4) {
+    bool sm = false;                          // SM teams (uniform length only)
+    const bool sm_able = !lens && (D == 64 ? sm_team_ok<64>() : sm_team_ok<128>());
+    if (num_splits == LMO_SPLITS_SMTEAM) {
+        a.num_splits = num_splits = 0;
+        sm = sm_able;
+        if (!sm) a.team = choose_team(pairs, (int64_t)max_ctas * kWarps);
+    } else if (num_splits == LMO_SPLITS_STREAMK) {
+        a.num_splits = num_splits = 0;        // explicit stream-K
+    } else if (num_splits == 1 || num_splits == 2 || num_splits == 4) {
         a.team = num_splits;                  // explicit team size (batch-independent results)
         a.num_splits = 0;
     } else if (num_splits == 0) {
         a.team = choose_team(pairs, (int64_t)max_ctas * kWarps);
-        static const char *sched = getenv("LMO_ATTN_SCHED");   // experiments: streamk | team1|2|4
-        if (sched && sched[0] == 's') a.team = 0;
+        static const char *sched = getenv("LMO_ATTN_SCHED");   // experiments: streamk | sm | team1|2|4
+        if (sched && !strcmp(sched, "streamk")) a.team = 0;
+        if (sched && !strcmp(sched, "sm") && sm_able) { a.team = 0; sm = true; }
         if (sched && sched[0] == 't') a.team = atoi(sched + 4);
     }
-    if (a.k_new && !a.team) {
-        // no pair teams (stream-K / fixed splits): append with its own kernel first
+    if (a.k_new && !a.team && (lens || a.num_splits > 0)) {
+        // fixed splits, or stream-K over per-sequence lengths: append with its own kernel first
         const cudaError_t e = launch_kv_append(c, k_new, v_new, 1, len - 1, lens, st, /*pos_from_lens=*/1);
         if (e != cudaSuccess) return e;
         a.k_new = a.v_new = nullptr;
@@ -1430,13 +1632,15 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     if (ctas < 1) ctas = 1;
     static const char *cap_env = getenv("LMO_ATTN_MAX_CTAS");   // tuning / experiments only
     if (cap_env && atoi(cap_env) > 0 && ctas > atoi(cap_env)) ctas = atoi(cap_env);
+    const int NW = sm ? kSmWarps : kWarps;
+    if (sm) ctas = device_sm_count();
     {   // the work map (uniform-length fields; per-sequence ones are completed on device)
         WorkMap &wm = a.wm;
         wm.prefix = nullptr;
         wm.B = c.batch;
         wm.Hkv = c.kv_heads;
         wm.k = a.num_splits;
-        wm.W = (int)ctas * kWarps;
+        wm.W = (int)ctas * NW;
         wm.nbu = lens ? 0 : (int)nbu;
         wm.N = lens ? 0 : (int)(pairs * nbu);
         wm.V = wm.k == 0 ? (wm.N < wm.W ? wm.N : wm.W) : (int)pairs * wm.k;
@@ -1444,11 +1648,17 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
         wm.n_teams = a.team ? wm.W / a.team : 0;
         wm.tsh = a.team == 4 ? 2 : a.team == 2 ? 1 : 0;
         wm.dHkv = FastDiv((uint32_t)c.kv_heads);
+        wm.sm = sm ? 1 : 0;
+        wm.P = (int)pairs;
+        wm.C = (int)ctas;
+        wm.NW = NW;
+        if (sm) wm.V = wm.W;
     }
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)ctas);
-    cfg.blockDim = dim3(kWarps * 32);
-    cfg.dynamicSmemBytes = D == 64 ? smem_bytes<64>(Bp) : smem_bytes<128>(Bp);
+    cfg.blockDim = dim3(NW * 32);
+    cfg.dynamicSmemBytes = sm ? (D == 64 ? smem_bytes<64, kSmWarps>(0) : smem_bytes<128, kSmWarps>(0))
+                              : (D == 64 ? smem_bytes<64>(Bp) : smem_bytes<128>(Bp));
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
@@ -1456,10 +1666,17 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     const bool mha = a.G == 1;
-    cudaError_t e = D == 64 ? (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, true>, a)
-                                   : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false>, a))
-                            : (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, true>, a)
-                                   : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, false>, a));
+    cudaError_t e;
+    if (sm)
+        e = D == 64 ? (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, true, kSmWarps>, a)
+                           : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false, kSmWarps>, a))
+                    : (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, true, kSmWarps>, a)
+                           : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, false, kSmWarps>, a));
+    else
+        e = D == 64 ? (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, true, kWarps>, a)
+                           : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false, kWarps>, a))
+                    : (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, true, kWarps>, a)
+                           : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, false, kWarps>, a));
     if (e != cudaSuccess) return e;
     note_launch();
     return cudaGetLastError();

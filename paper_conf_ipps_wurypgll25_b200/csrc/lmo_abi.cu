@@ -109,7 +109,7 @@ lmo_status lmo_kv_append_quant(const lmo_kv_cache *cache, const void *k_new, con
 
 size_t lmo_decode_attention_workspace_bytes(int32_t batch, int32_t kv_heads, int32_t q_heads,
                                             int32_t head_dim, int32_t num_splits) {
-    if (batch <= 0 || kv_heads <= 0 || q_heads <= 0 || q_heads % kv_heads != 0 || num_splits < 0 ||
+    if (batch <= 0 || kv_heads <= 0 || q_heads <= 0 || q_heads % kv_heads != 0 || num_splits < LMO_SPLITS_SMTEAM ||
         (head_dim != 64 && head_dim != 128))
         return 0;
     return attn_workspace_bytes(batch, kv_heads, q_heads, head_dim, num_splits);
@@ -124,7 +124,7 @@ static lmo_status check_attention(const lmo_kv_cache *cache, const void *q, int3
     if (!q || !out) return LMO_ERR_NULL;
     if (q_heads <= 0 || q_heads % cache->kv_heads != 0) return LMO_ERR_SHAPE;
     if (q_heads / cache->kv_heads > 8) return LMO_ERR_UNSUPPORTED;
-    if (num_splits < 0) return LMO_ERR_SHAPE;
+    if (num_splits < LMO_SPLITS_SMTEAM) return LMO_ERR_SHAPE;
     if (out_dtype != LMO_F16 && out_dtype != LMO_F32) return LMO_ERR_UNSUPPORTED;
     if (!seq_lens_dev && (len < 1 || len > cache->capacity)) return LMO_ERR_SHAPE;
     if (seq_lens_dev && cache->batch > 1024) return LMO_ERR_UNSUPPORTED;

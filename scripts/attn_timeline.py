@@ -73,3 +73,24 @@ print("smsp index histogram:", sorted(collections.Counter(sp.tolist()).items()))
 for k in sorted(set(cnt_sp.values())):
     m = torch.tensor([cnt_sp[(a, c)] == k for a, c in zip(sm.tolist(), sp.tolist())])
     print(f"  warps on SMSPs holding {k} busy warps: {int(m.sum())}, end median {end[m].median():.2f} max {end[m].max():.2f} us")
+
+# per-warp breakdown (launch 2): data->end vs segments, mbarrier wait share
+segs = (b[:, 3].long() & 0xffff)
+dte = (b[:, 7] - b[:, 6]) / 1e3
+wait_us = b[:, 0] / 1.965e3
+print("data->end by segments/warp:")
+for k in sorted(set(segs.tolist())):
+    m = segs == k
+    print(f"  segs={k}: warps {int(m.sum())}, data->end median {dte[m].median():.2f} max {dte[m].max():.2f} us, "
+          f"mbar wait median {wait_us[m].median():.2f} us")
+slow = dte > dte.median() + 5
+print(f"slow warps (>median+5us): {int(slow.sum())}, their wait median {wait_us[slow].median() if slow.any() else 0:.2f} us, "
+      f"end-1st-data median {dte[slow].median() if slow.any() else 0:.2f}")
+cs = (b[:, 15].long() & 0xffffffff).double() / 1.965e3
+ce = (b[:, 15].long() >> 32).double() / 1.965e3
+for k in sorted(set(segs.tolist())):
+    m = segs == k
+    print(f"  segs={k}: seg-start section median {cs[m].median():.2f} us, seg-end section median {ce[m].median():.2f} max {ce[m].max():.2f} us")
+le = (b[:, 13] - b[:, 4].min()) / 1e3
+z2 = (b[:, 7] - b[:, 4].min()) / 1e3
+print(f"launch 2 (rel. to first entry): loop end {le.min():.2f}/{le.median():.2f}/{le.max():.2f}  kernel exit {z2.min():.2f}/{z2.median():.2f}/{z2.max():.2f} us")

@@ -9,7 +9,15 @@ from paper_conf_ipps_wurypgll25_b200 import lmo
 from paper_conf_ipps_wurypgll25_b200.configs import CONFIGS, attention_launch_bytes
 
 keys = [a for a in sys.argv[1:] if not a.startswith('-')] or ["c2"]
+# custom shape: SHAPE=B,Hkv,G,L (head_dim 128) replaces the config list
+if os.environ.get("SHAPE"):
+    import dataclasses
+    B_, H_, G_, L_ = [int(x) for x in os.environ["SHAPE"].split(",")]
+    CONFIGS = dict(CONFIGS)
+    CONFIGS["custom"] = dataclasses.replace(CONFIGS["c2"], batch=B_, kv_heads=H_, q_heads=H_ * G_, prompt=L_, gen=2)
+    keys = ["custom"]
 reps = int(os.environ.get("REPS", "10"))
+splits = int(os.environ.get("SPLITS", "0"))
 for key in keys:
     w = CONFIGS[key]
     L = int(os.environ.get("LEN", "0")) or (w.prompt + w.gen // 2)
@@ -25,13 +33,13 @@ for key in keys:
     kn = torch.randn(w.batch, w.kv_heads, w.head_dim, device='cuda').half()
     vn = torch.randn_like(kn)
     out = torch.empty(w.batch, w.q_heads, w.head_dim, device='cuda')
-    ws = lmo.attention_workspace(w.batch, w.kv_heads, w.q_heads, w.head_dim, 0)
+    ws = lmo.attention_workspace(w.batch, w.kv_heads, w.q_heads, w.head_dim, splits)
     abis = [c.abi() for c in caches]
     st = torch.cuda.Stream()
     def layers():
         for l in range(nl):
             lmo.lmo_decode_step_q4(caches[l], kn, vn, q, L, out=out, workspace=ws, abi=abis[l],
-                                   flags=lmo.LMO_STEP_CACHE_STABLE, stream=st)
+                                   flags=lmo.LMO_STEP_CACHE_STABLE, stream=st, num_splits=splits)
     with torch.cuda.stream(st):
         layers()
     torch.cuda.synchronize()

@@ -210,6 +210,9 @@ CASES = [  # (B, Hkv, G, d, L, num_splits)
     (3, 5, 1, 128, 100, 3), (2, 2, 8, 64, 1000, 0), (1, 3, 1, 128, 1000, 7), (2, 1, 8, 128, 4090, 0),
     (5, 7, 3, 128, 333, 0), (1, 1, 1, 128, 1, 4), (64, 8, 1, 128, 40, 0), (3, 4, 2, 128, 517, 2),
     (2, 3, 8, 128, 250, 4), (3, 2, 1, 64, 47, 2),
+    (3, 5, 1, 128, 100, -1), (2, 2, 8, 128, 65, -1), (64, 8, 1, 128, 40, -1), (2, 3, 2, 64, 333, -1),
+    (3, 5, 1, 128, 100, -2), (2, 2, 8, 128, 65, -2), (64, 8, 1, 128, 40, -2), (2, 3, 2, 64, 333, -2),
+    (1, 1, 1, 128, 1000, -2), (40, 9, 1, 128, 77, -2), (5, 3, 8, 128, 1, -2), (300, 4, 1, 64, 20, -2),
 ]
 
 
@@ -319,7 +322,12 @@ def test_full_size_sampled_rows(lmo, key):
 @pytest.mark.parametrize("B,Hkv,G,d,L,ns", [(4, 6, 1, 128, 300, 0), (2, 2, 8, 128, 129, 0),
                                             (3, 4, 2, 64, 77, 2), (2, 3, 1, 128, 40, 4),
                                             (2, 2, 4, 128, 200, 3), (1, 2, 1, 128, 1, 0),
-                                            (3, 5, 1, 128, 33, 0), (2, 2, 8, 128, 16, 0)])
+                                            (3, 5, 1, 128, 33, 0), (2, 2, 8, 128, 16, 0),
+                                            (4, 6, 1, 128, 300, -1), (3, 4, 8, 128, 129, -1),
+                                            (5, 3, 1, 64, 77, -1), (2, 3, 1, 128, 1, -1),
+                                            (7, 5, 2, 128, 47, -1), (4, 6, 1, 128, 300, -2),
+                                            (3, 4, 8, 128, 129, -2), (5, 3, 1, 64, 77, -2),
+                                            (2, 3, 1, 128, 1, -2), (64, 9, 1, 128, 47, -2)])
 def test_decode_step_fused_append(lmo, B, Hkv, G, d, L, ns, flags):
     """lmo_decode_step_q4 == append(new token at L-1) then attention over L, for the
     team schedule (one launch) and the stream-K fallback (two launches)."""

@@ -45,6 +45,7 @@ def parse():
     p.add_argument("--splits", type=int, default=0, help="num_splits (0 = stream-K auto)")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-stream", action="store_true", help="skip the A1/A5 weight streaming leg")
+    p.add_argument("--no-offload", action="store_true", help="skip the host-offloaded KV leg")
     p.add_argument("--no-early", action="store_true", help="disable LMO_STEP_CACHE_STABLE")
     p.add_argument("--cpu-sample-seconds", type=float, default=10.0)
     return p.parse_args()
@@ -397,6 +398,54 @@ def run_ours(args):
                          "peak": peak, **res}
             del xw, codes, meta, yw
 
+    # ---- NEXT-4 leg: the same decode step with every layer's q4 cache offloaded to pinned
+    # host memory (the paper's setting, Alg 1): per layer a strided H2D of the old rows
+    # into a 3-slot device ring, the fused step, a D2H of the new row (lmo_offload_*).
+    offload = None
+    host_bytes = nl * caches[0].nbytes()
+    if not args.no_offload and host_bytes <= 8e9:
+        ox = lmo.OffloadKV(nl, B, Hkv, w.capacity, d, slots=3, device=dev)
+        for l in range(nl):
+            ox.host_layer(l).copy_(caches[l].kv.cpu())
+        t = t_mid
+        L = s + t
+        oout = torch.empty((nl, B, Hq, d), dtype=torch.float32, device=dev)
+        kq = qbuf[t].view(nl, B, Hq, d)
+        with torch.cuda.stream(stream):
+            ox.decode_step(kbuf[t], vbuf[t], kq, L, softmax_scale=sigma, num_splits=args.splits,
+                           out=oout, workspace=ws, stream=stream)
+            o0, o1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            o0.record(stream)
+            nrep = 3
+            for _ in range(nrep):
+                ox.decode_step(kbuf[t], vbuf[t], kq, L, softmax_scale=sigma, num_splits=args.splits,
+                               out=oout, workspace=ws, stream=stream)
+            o1.record(stream)
+        o1.synchronize()
+        off_ms = reduce_max(o0.elapsed_time(o1)) / nrep
+        # raw pinned H2D bandwidth of this box (one 1 GiB copy) for the fraction
+        hb = torch.empty(1 << 30, dtype=torch.uint8).pin_memory()
+        db = torch.empty(1 << 30, dtype=torch.uint8, device=dev)
+        db.copy_(hb, non_blocking=True)
+        torch.cuda.synchronize()
+        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        p0.record()
+        db.copy_(hb, non_blocking=True)
+        p1.record()
+        p1.synchronize()
+        pcie = (1 << 30) / (p0.elapsed_time(p1) / 1e3) / 1e9
+        del hb, db
+        h2d_step = nl * B * Hkv * (L - 1) * lmo.row_bytes(d)
+        offload = {"value": world * B / (off_ms / 1e3), "unit": "tokens/s", "ms_per_step": off_ms,
+                   "L": L, "ring_slots": 3, "host_bytes": host_bytes,
+                   "h2d_bytes_per_step": h2d_step,
+                   "d2h_bytes_per_step": nl * B * Hkv * lmo.row_bytes(d),
+                   "h2d_gbs": h2d_step / (off_ms / 1e3) / 1e9, "h2d_peak_gbs_measured": pcie,
+                   "frac_of_h2d_peak": h2d_step / (off_ms / 1e3) / 1e9 / pcie,
+                   "path": "pinned host q4 caches -> strided H2D (copy stream) -> fused step on a ring slot -> D2H of the new row"}
+        ox.close()
+        del ox, oout
+
     # ---- e2e: host buffers, H2D of each step's inputs + D2H of its result in the region
     e2e = None
     if not args.no_e2e:
@@ -481,6 +530,7 @@ def run_ours(args):
                          "per_launch_us": attn_ms * 1e3, "algorithmic_bytes_per_launch": attn_bytes},
             "prefill_ms_all_layers": pre_ms,
             "streaming": streaming,
+            "offload": offload,
             "gpu_launches": launches_per_step * args.steps,
             "clocks": clocks,
             "e2e": e2e,

@@ -197,6 +197,49 @@ lmo_status lmo_decode_step_q4(const lmo_kv_cache *cache, const void *k_new_f16,
                               int32_t num_splits, void *out, lmo_dtype out_dtype, void *workspace,
                               size_t workspace_bytes, uint32_t flags, void *stream);
 
+/* ---------------------------------------------------------------------------
+ * NEXT-4: host-offloaded q4 KV cache -- the paper's setting.
+ * LM-Offload keeps the KV cache in CPU memory and, per layer, loads the cache
+ * to the GPU, computes, and stores the new token's K/V back, overlapping the
+ * loads of the next layers with the current layer's compute (Alg 1,
+ * load_cache / compute / store_cache; Eq 6-7).
+ *
+ * host_kv   : pinned host memory (caller-owned, e.g. cudaHostAlloc or
+ *             torch pin_memory), `layers` consecutive q4 caches each laid out
+ *             exactly like a device lmo_kv_cache: [B][Hkv][cap][row] bytes.
+ *             `shape` gives B, Hkv, cap, head_dim (its kv field is ignored).
+ * ring_dev  : device staging ring, caller-owned, >= lmo_offload_ring_bytes();
+ *             slot s is a full device cache of the same shape.
+ * ring_slots: >= 1; layer l uses slot l % ring_slots, so up to ring_slots - 1
+ *             layers are loaded ahead of the one being computed.
+ * The executor owns two copy streams (H2D, D2H) and per-slot events; it never
+ * allocates device memory.  Destroy with lmo_offload_destroy.
+ * ------------------------------------------------------------------------- */
+typedef struct lmo_offload *lmo_offload_t;
+size_t lmo_offload_ring_bytes(const lmo_kv_cache *shape, int32_t ring_slots);
+lmo_status lmo_offload_create(const lmo_kv_cache *shape, int32_t layers, uint8_t *host_kv,
+                              uint8_t *ring_dev, int32_t ring_slots, lmo_offload_t *out);
+
+/* One decode step of all layers at length L = len (the new token goes to slot
+ * len-1 of every layer's cache).  For each layer l:
+ *   H2D   rows [0, len-1) of every (b, kvh) of host layer l -> ring slot
+ *         (one strided copy; waits until the slot's previous user is stored),
+ *   A2-A4 lmo_decode_step_q4 on the slot with k_new/v_new/q of layer l
+ *         (on compute_stream, after the H2D),
+ *   D2H   row len-1 of every (b, kvh) of the slot -> host layer l.
+ * k_new, v_new : device [layers][B][Hkv][head_dim] fp16; q device
+ * [layers][B][q_heads][head_dim] fp16; out device [layers][B][q_heads][head_dim]
+ * (out_dtype).  Other arguments as lmo_decode_step_q4 (num_splits, workspace).
+ * Enqueues only; compute_stream is made to wait for the last D2H, so a
+ * synchronize on compute_stream covers the whole step.  Host-side argument
+ * errors are reported before anything is enqueued. */
+lmo_status lmo_offload_decode_step(lmo_offload_t ex, const void *k_new_f16, const void *v_new_f16,
+                                   const void *q_f16, int32_t q_heads, int32_t len,
+                                   float softmax_scale, int32_t num_splits, void *out,
+                                   lmo_dtype out_dtype, void *workspace, size_t workspace_bytes,
+                                   void *compute_stream);
+lmo_status lmo_offload_destroy(lmo_offload_t ex);
+
 /* Human-readable name of a status code (static string). */
 const char *lmo_status_string(lmo_status status);
 

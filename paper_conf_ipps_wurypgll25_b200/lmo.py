@@ -56,6 +56,15 @@ def _load():
         f = getattr(L, name)
         f.argtypes = args
         f.restype = ctypes.c_int
+    L.lmo_offload_ring_bytes.argtypes = [ctypes.POINTER(lmo_kv_cache), i32]
+    L.lmo_offload_ring_bytes.restype = ctypes.c_size_t
+    L.lmo_offload_create.argtypes = [ctypes.POINTER(lmo_kv_cache), i32, P, P, i32, ctypes.POINTER(P)]
+    L.lmo_offload_create.restype = ctypes.c_int
+    L.lmo_offload_decode_step.argtypes = [P, P, P, P, i32, i32, ctypes.c_float, i32, P, ctypes.c_int,
+                                          P, ctypes.c_size_t, P]
+    L.lmo_offload_decode_step.restype = ctypes.c_int
+    L.lmo_offload_destroy.argtypes = [P]
+    L.lmo_offload_destroy.restype = ctypes.c_int
     L.lmo_decode_attention_workspace_bytes.argtypes = [i32, i32, i32, i32, i32]
     L.lmo_decode_attention_workspace_bytes.restype = ctypes.c_size_t
     L.lmo_status_string.argtypes = [ctypes.c_int]
@@ -75,7 +84,9 @@ EXPORTS = ["lmo_quantize_groupwise", "lmo_dequantize_groupwise", "lmo_kv_append_
            "lmo_kv_row_bytes",
            "lmo_decode_attention_workspace_bytes", "lmo_decode_attention_q4", "lmo_decode_step_q4",
            "lmo_status_string",
-           "lmo_gen_fill_f16", "lmo_launch_count", "lmo_version"]
+           "lmo_gen_fill_f16", "lmo_launch_count", "lmo_version",
+           "lmo_offload_ring_bytes", "lmo_offload_create", "lmo_offload_decode_step",
+           "lmo_offload_destroy"]
 
 
 def _check(status: int, fn: str) -> None:
@@ -272,3 +283,70 @@ def lmo_gen_fill_f16(dst: torch.Tensor, seed: int, stream_id: int, layer: int, b
     _check(_lib.lmo_gen_fill_f16(_ptr(dst), nb, nh, npos, dim, seed, stream_id, layer, b0, h0, p0,
                                  group, _stream(stream)), "lmo_gen_fill_f16")
     return dst
+
+
+# ------------------------------------------------------- NEXT-4: offloaded KV
+
+class OffloadKV:
+    """Host-offloaded q4 KV caches of `layers` layers (pinned host memory, the
+    paper's setting) + a device staging ring of `slots` layer caches, driven by
+    the library's executor (lmo_offload_*).  Layout of each host layer =
+    KVCache.kv ([B][Hkv][cap][row] bytes)."""
+
+    def __init__(self, layers: int, batch: int, kv_heads: int, capacity: int, head_dim: int,
+                 slots: int = 2, device="cuda"):
+        cap = (capacity + 15) // 16 * 16
+        self.layers, self.batch, self.kv_heads, self.capacity, self.head_dim = \
+            layers, batch, kv_heads, cap, head_dim
+        self.shape = lmo_kv_cache(None, batch, kv_heads, cap, head_dim)
+        self.row = row_bytes(head_dim)
+        self.layer_bytes = batch * kv_heads * cap * self.row
+        self.host = torch.empty(layers * self.layer_bytes, dtype=torch.uint8).pin_memory()
+        n = _lib.lmo_offload_ring_bytes(ctypes.byref(self.shape), slots)
+        if n == 0:
+            raise LmoError(LMO_ERR_SHAPE, "lmo_offload_ring_bytes")
+        self.ring = torch.empty(n, dtype=torch.uint8, device=device)
+        self._h = ctypes.c_void_p()
+        _check(_lib.lmo_offload_create(ctypes.byref(self.shape), layers,
+                                       ctypes.c_void_p(self.host.data_ptr()),
+                                       ctypes.c_void_p(self.ring.data_ptr()), slots,
+                                       ctypes.byref(self._h)), "lmo_offload_create")
+
+    def host_layer(self, l: int) -> torch.Tensor:
+        """View of host layer l as [B][Hkv][cap][row] uint8."""
+        return self.host[l * self.layer_bytes:(l + 1) * self.layer_bytes].view(
+            self.batch, self.kv_heads, self.capacity, self.row)
+
+    def decode_step(self, k_new: torch.Tensor, v_new: torch.Tensor, q: torch.Tensor, length: int,
+                    softmax_scale: float | None = None, num_splits: int = 0,
+                    out: torch.Tensor | None = None, out_dtype: torch.dtype = torch.float32,
+                    workspace: torch.Tensor | None = None, stream=None) -> torch.Tensor:
+        """All layers' decode step at L = length: k_new/v_new [layers][B][Hkv](1)[d],
+        q [layers][B][Hq](1)[d] -> out [layers][B][Hq][d]."""
+        nl, B = self.layers, self.batch
+        Hq = q.shape[2]
+        d = self.head_dim
+        if softmax_scale is None:
+            softmax_scale = 1.0 / math.sqrt(d)
+        if out is None:
+            out = torch.empty((nl, B, Hq, d), dtype=out_dtype, device=q.device)
+        if workspace is None:
+            workspace = attention_workspace(B, self.kv_heads, Hq, d, num_splits, q.device)
+        _need_cuda(k_new, v_new, q, out, workspace)
+        dt = LMO_F16 if out.dtype == torch.float16 else LMO_F32
+        _check(_lib.lmo_offload_decode_step(self._h, _ptr(k_new), _ptr(v_new), _ptr(q), Hq, length,
+                                            float(softmax_scale), num_splits, _ptr(out), dt,
+                                            _ptr(workspace), workspace.numel(), _stream(stream)),
+               "lmo_offload_decode_step")
+        return out
+
+    def close(self):
+        if self._h:
+            _lib.lmo_offload_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -89,3 +89,21 @@ def test_binding_has_no_cpu_fallback():
             if f.endswith((".py", ".cu", ".cuh", ".h")):
                 txt = open(os.path.join(dirpath, f)).read()
                 assert not bad.search(txt), f
+
+
+def test_offload_validation_without_gpu(lib):
+    import ctypes
+    L = lib._lib
+    good = lib.lmo_kv_cache(None, 2, 2, 32, 128)
+    bad = lib.lmo_kv_cache(None, 2, 2, 32, 96)
+    assert L.lmo_offload_ring_bytes(ctypes.byref(good), 2) == 2 * 2 * 2 * 32 * 144
+    assert L.lmo_offload_ring_bytes(ctypes.byref(bad), 2) == 0
+    assert L.lmo_offload_ring_bytes(ctypes.byref(good), 0) == 0
+    h = ctypes.c_void_p()
+    P = ctypes.c_void_p
+    assert L.lmo_offload_create(ctypes.byref(good), 0, P(4096), P(4096), 2, ctypes.byref(h)) == lib.LMO_ERR_SHAPE
+    assert L.lmo_offload_create(ctypes.byref(good), 2, None, P(4096), 2, ctypes.byref(h)) == lib.LMO_ERR_NULL
+    assert L.lmo_offload_create(ctypes.byref(good), 2, P(4100), P(4096), 2, ctypes.byref(h)) == lib.LMO_ERR_ALIGN
+    assert L.lmo_offload_decode_step(None, P(16), P(16), P(16), 2, 5, 1.0, 0, P(16), 1, P(16), 1 << 20, None) \
+        == lib.LMO_ERR_NULL
+    assert L.lmo_offload_destroy(None) == lib.LMO_ERR_NULL

@@ -50,6 +50,15 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_LAZY_MAX
 #define LMO_LAZY_MAX 0   // measured: no gain (c2), 3% loss (c5 GQA)
 #endif
+#ifndef LMO_Q_PF_L1
+#define LMO_Q_PF_L1 0    // next segment's q rows: prefetch into L1 (1) or L2 (0)
+#endif
+#ifndef LMO_FENCE_CTA
+#define LMO_FENCE_CTA 0  // mbarrier init made visible to the async proxy with a CTA-scope fence
+#endif
+#ifndef LMO_NO_SCH
+#define LMO_NO_SCH 0     // 1: every schedule runs the generic kernel instance (experiments)
+#endif
 #ifndef LMO_ATTN_MINBLOCKS
 #define LMO_ATTN_MINBLOCKS 4
 #endif
@@ -183,15 +192,17 @@ struct SegIter {
         wm.decode(x, b, kvh, blk, nb);
     }
     // team mode: v = pair index, x0 = rank of this warp in its team (inline: cheap)
+    template <int SCH>
     __device__ __forceinline__ void team_seg(const WorkMap &wm) {
         if (v >= wm.B * wm.Hkv) {
             done = true;
             return;
         }
-        b = v / wm.Hkv;
+        b = (int)wm.dHkv.div((uint32_t)v);
         kvh = v - b * wm.Hkv;
         nb = wm.seq_nb(b);
-        const int lo = x0 * nb / wm.T, hi = (x0 + 1) * nb / wm.T;
+        const int T = SCH == 1 ? 1 : wm.T;
+        const int lo = SCH == 1 ? 0 : x0 * nb / T, hi = SCH == 1 ? nb : (x0 + 1) * nb / T;
         blk = lo;
         sn = hi - lo;
         sx = wm.seq_start(b) + kvh * nb + lo;
@@ -213,9 +224,10 @@ struct SegIter {
         a += sn;
         done = false;
     }
+    template <int SCH>
     __device__ __forceinline__ void begin_v(const WorkMap &wm) {
-        if (wm.T) {
-            team_seg(wm);
+        if (SCH != 0 || wm.T) {
+            team_seg<SCH>(wm);
         } else if (wm.sm) {
             x0 = wm.R(v);
             x1 = wm.R(v + 1);
@@ -250,10 +262,11 @@ struct SegIter {
         done = true;
     }
     // out of line: runs only at segment transitions, keeps the hot loop small (I-cache)
+    template <int SCH>
     __device__ __forceinline__ void next(const WorkMap &wm) {
-        if (wm.T) {
+        if (SCH != 0 || wm.T) {
             v += wm.n_teams;
-            team_seg(wm);
+            team_seg<SCH>(wm);
         } else if (wm.sm) {
             sm_seg(wm);
         } else {
@@ -415,11 +428,11 @@ struct WarpCtl {
 
 // Producer segment setup (out of line): skip empty segments, then the byte cursor
 // of the new segment's tokens < L.
-template <int D>
+template <int D, int SCH>
 __device__ __noinline__ void prod_seg(WarpCtl &ctl, const WorkMap &wm, const uint8_t *kv,
                                      const int32_t *lens, int cap, int len) {
     SegIter &pc = ctl.pc;
-    while (!pc.done && pc.sn == 0) pc.next(wm);
+    while (!pc.done && pc.sn == 0) pc.template next<SCH>(wm);
     if (pc.done) {
         ctl.pdone = 1;
         return;
@@ -442,9 +455,13 @@ struct KState {       // per-stage scores handed from the K part to the V part
 template <int NW>
 __host__ __device__ constexpr int bars_bytes() { return (NW * kStages * 8 + 127) / 128 * 128; }
 
-template <int D, bool MHA, int NW>
+// SCH: 0 = any schedule (runtime work map mode); 1 = pair teams with T = 1 (one warp
+// per pair, the default); 2 = pair teams with T > 1.  The specialised instances drop
+// the other modes' code (smaller kernel: fewer cold instruction-cache misses).
+template <int D, bool MHA, int NW, int SCH = 0>
 __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1) decode_attn_q4_kernel(const AttnArgs a) {
     using GG = Geo<D>;
+    constexpr bool TEAMK = SCH != 0;
     constexpr int NG = GG::NG;
     extern __shared__ __align__(128) uint8_t smem[];
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem);                 // [NW][kStages]
@@ -499,7 +516,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
     }
     if (threadIdx.x == 0) {
         WorkMap wm = a.wm;
-        if (wm.sm) {
+        if (SCH == 0 && wm.sm) {
             const int p0 = (int)((long long)blockIdx.x * wm.P / wm.C);
             const int p1 = (int)((long long)(blockIdx.x + 1) * wm.P / wm.C);
             wm.vb = blockIdx.x * wm.NW;
@@ -548,8 +565,8 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
         ctl.psrc += kStageTok * GG::ROW;
         ctl.ptok += kStageTok;
         if (ctl.ptok >= ctl.pend) {
-            ctl.pc.next(wms);
-            prod_seg<D>(ctl, wms, a.kv, a.lens, a.cap, a.len);
+            ctl.pc.template next<SCH>(wms);
+            prod_seg<D, SCH>(ctl, wms, a.kv, a.lens, a.cap, a.len);
         }
     };
 
@@ -565,23 +582,24 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
     auto prologue = [&](bool before_append) {   // (always called with true)
         if (lane == 0) {
             for (int s = 0; s < kStages; ++s) mbar_init(&wbar[s], 1);
-            fence_mbar_init();
+            if (LMO_FENCE_CTA) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+            else fence_mbar_init();
 #if LMO_ATTN_PROFILE
             prof_gf = gtimer();
 #endif
-            if (wms.T) {
+            if (TEAMK || wms.T) {
                 // team ids interleaved across CTAs (tau = team-in-CTA * grid + CTA): the busy
                 // teams spread evenly over the SMs when there are fewer pairs than teams
-                ctl.cc.v = (warp / wms.T) * gridDim.x + blockIdx.x;   // team id = first pair
-                ctl.cc.x0 = warp % wms.T;                             // rank in team
+                ctl.cc.v = (SCH == 1 ? warp : warp / wms.T) * gridDim.x + blockIdx.x;   // team id = first pair
+                ctl.cc.x0 = SCH == 1 ? 0 : warp % wms.T;                              // rank in team
             } else {
                 ctl.cc.v = gw;
             }
-            ctl.cc.begin_v(wms);
+            ctl.cc.template begin_v<SCH>(wms);
             ctl.pc = ctl.cc;
             ctl.qb = -1;
             ctl.qkvh = -1;
-            prod_seg<D>(ctl, wms, a.kv, a.lens, a.cap, a.len);
+            prod_seg<D, SCH>(ctl, wms, a.kv, a.lens, a.cap, a.len);
 #if LMO_ATTN_PROFILE
             prof_gb = gtimer();
 #endif
@@ -653,9 +671,9 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
     bool app_warp = false;
     int app_lo = 0, app_hi = 0, app_step = 1;
     if (a.k_new) {
-        if (wms.T) {
-            app_warp = (gw % wms.T) == wms.T - 1;
-            app_lo = (warp / wms.T) * gridDim.x + blockIdx.x;
+        if (TEAMK || wms.T) {
+            app_warp = SCH == 1 ? true : (gw % wms.T) == wms.T - 1;
+            app_lo = (SCH == 1 ? warp : warp / wms.T) * gridDim.x + blockIdx.x;
             app_hi = a.B * a.Hkv;
             app_step = wms.n_teams;
         } else if (gw < wms.V) {
@@ -666,8 +684,9 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
     }
     const int lane8 = lane & 7, kvsel = lane / (8 * NG), grp8 = (lane >> 3) % NG;
     const bool lane_ok = lane < 16 * NG;
-    const int p_first = wms.T ? (warp / wms.T) * gridDim.x + blockIdx.x : 0;
-    bool first_ok = wms.T && p_first < a.B * a.Hkv;
+    const int p_first = SCH == 1 ? warp * gridDim.x + blockIdx.x
+                                 : (TEAMK || wms.T) ? (warp / wms.T) * gridDim.x + blockIdx.x : 0;
+    bool first_ok = (TEAMK || wms.T) && p_first < a.B * a.Hkv;
     int fb = 0, fk = 0;                 // pair of the warp's first segment (q prefetch)
     auto app_src = [&](int p) {
         return (kvsel == 0 ? a.k_new : a.v_new) + (int64_t)p * D + grp8 * 64 + lane8 * 8;
@@ -680,7 +699,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
     auto fetch_first = [&]() {
         if (app_warp && lane_ok && app_lo < app_hi)
             xv_first = *reinterpret_cast<const uint4 *>(app_src(app_lo));
-        if (wms.T) {
+        if (TEAMK || wms.T) {
             fb = (int)wms.dHkv.div((uint32_t)p_first);
             fk = p_first - fb * a.Hkv;
         } else {                        // stream-K / SM teams: set by the producer prologue
@@ -727,7 +746,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
         prologue(true);
         asm volatile("griddepcontrol.wait;\n" ::: "memory");
         fetch_first();
-    } else if (!wms.T) {
+    } else if (!(TEAMK || wms.T)) {
         prologue(true);
         fetch_first();
     } else {
@@ -784,7 +803,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
             d.v = cc.v; d.x0 = cc.x0;
             d.L = a.lens ? min(a.lens[cc.b], a.cap) : a.len;
             ctl.seg = d;
-            cc.next(wms);
+            cc.template next<SCH>(wms);
         }
         __syncwarp();
         const int seg_n = ctl.seg.sn, blk0 = ctl.seg.blk0, L = ctl.seg.L;
@@ -813,7 +832,8 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
             const char *qn = reinterpret_cast<const char *>(a.q + ((int64_t)nb_ * a.Hq + nk_ * a.G + lane) * D);
 #pragma unroll
             for (int o = 0; o < D * 2; o += 128)
-                asm volatile("prefetch.global.L2 [%0];" ::"l"(qn + o));
+                if (LMO_Q_PF_L1) asm volatile("prefetch.global.L1 [%0];" ::"l"(qn + o));
+                else asm volatile("prefetch.global.L2 [%0];" ::"l"(qn + o));
         }
 
         float m_run[2] = {NEG_INF, NEG_INF};
@@ -1176,8 +1196,8 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
                 }
         const SegDesc sd = ctl.seg;
         const int64_t rowbase = (int64_t)sd.b * a.Hq + (int64_t)sd.kvh * a.G;
-        const bool full = (sd.blk0 == 0) && (sd.sn == sd.nb) && wms.T <= 1;
-        if (wms.T > 1) {
+        const bool full = SCH == 1 || (SCH == 0 && (sd.blk0 == 0) && (sd.sn == sd.nb) && wms.T <= 1);
+        if (SCH == 2 || (SCH == 0 && wms.T > 1)) {
             // ---- pair team: partials through L2 scratch, named barrier, rank 0 merges
             const int T = wms.T;
             const int64_t myslot = 2 * (int64_t)gw + (team_k & 1);
@@ -1266,7 +1286,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
                     if (h < a.G) store_row8<D>(a, rowbase + h, grp * 64 + 8 * g, vo[e][grp]);
                 }
             }
-        } else {
+        } else if constexpr (SCH == 0) {
             const WorkMap wm = wms;
             // pair start = global index of the pair's first block
             const int ps = wm.seq_start(sd.b) + sd.kvh * sd.nb;
@@ -1367,7 +1387,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
 #endif
     // ---- SM teams (A4): the CTA's pairs that were cut between warps are merged here,
     // once, after one CTA barrier (partials in L2 scratch; no fences or atomics).
-    if (wms.sm) {
+    if (SCH == 0 && wms.sm) {
         __syncthreads();
         const WorkMap wm = wms;
         const int c = blockIdx.x;
@@ -1517,9 +1537,13 @@ static int ctas_per_sm(int B_prefix) {   // (MHA and GQA variants have the same 
     if (dev < 0 || dev >= 64) dev = 0;
     const int mode = B_prefix > 0 ? 1 : 0;
     if (occ[dev][mode] == 0) {
-        for (int m = 0; m < 2; ++m)
-            cudaFuncSetAttribute(m ? decode_attn_q4_kernel<D, true, kWarps> : decode_attn_q4_kernel<D, false, kWarps>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem_bytes<D>(kMaxBatchSmem));
+        const int sz = (int)smem_bytes<D>(kMaxBatchSmem);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kWarps, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kWarps, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kWarps, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
         int n = 0, n1 = 0;
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n1, decode_attn_q4_kernel<D, true, kWarps>, kWarps * 32,
                                                       smem_bytes<D>(mode ? kMaxBatchSmem : 0));
@@ -1672,6 +1696,16 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false, kSmWarps>, a))
                     : (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, true, kSmWarps>, a)
                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, false, kSmWarps>, a));
+    else if (a.team == 1 && !LMO_NO_SCH)
+        e = D == 64 ? (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, true, kWarps, 1>, a)
+                           : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false, kWarps, 1>, a))
+                    : (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, true, kWarps, 1>, a)
+                           : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, false, kWarps, 1>, a));
+    else if (a.team > 1 && !LMO_NO_SCH)
+        e = D == 64 ? (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, true, kWarps, 2>, a)
+                           : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false, kWarps, 2>, a))
+                    : (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, true, kWarps, 2>, a)
+                           : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, false, kWarps, 2>, a));
     else
         e = D == 64 ? (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, true, kWarps>, a)
                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false, kWarps>, a))

@@ -37,7 +37,7 @@ class lmo_kv_cache(ctypes.Structure):
 
 
 def _load():
-    path = _build.LIB
+    path = os.environ.get("LMO_LIB") or _build.LIB   # LMO_LIB: alternate build (experiments)
     if not os.path.exists(path):
         raise ImportError(f"liblmo.so not built ({path}); run __graft_entry__.build()")
     L = ctypes.CDLL(path)

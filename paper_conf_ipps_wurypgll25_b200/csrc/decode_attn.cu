@@ -56,6 +56,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_FENCE_CTA
 #define LMO_FENCE_CTA 0  // mbarrier init made visible to the async proxy with a CTA-scope fence
 #endif
+#ifndef LMO_UNIFIED
+#define LMO_UNIFIED 1    // MHA: one masked loop body for every stage (0: separate FULL / GEN bodies)
+#endif
 #ifndef LMO_NO_SCH
 #define LMO_NO_SCH 0     // 1: every schedule runs the generic kernel instance (experiments)
 #endif
@@ -483,7 +486,10 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
 #endif
     asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory");
     const bool early = a.early && !a.lens;
-    if (!early) asm volatile("griddepcontrol.wait;\n" ::: "memory");
+    // per-sequence lengths may be produced by the previous kernel: wait first.  Uniform
+    // length: the work map and producer setup read only the launch arguments and run
+    // before the wait (they overlap the previous kernel's tail).
+    if (a.lens) asm volatile("griddepcontrol.wait;\n" ::: "memory");
 #if LMO_ATTN_PROFILE
     const unsigned long long prof_gw = gtimer();   // after the (non-early) wait
 #endif
@@ -579,7 +585,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
 #if LMO_ATTN_PROFILE
     unsigned long long prof_gf = 0, prof_gb = 0;
 #endif
-    auto prologue = [&](bool before_append) {   // (always called with true)
+    auto prologue_setup = [&]() {
         if (lane == 0) {
             for (int s = 0; s < kStages; ++s) mbar_init(&wbar[s], 1);
             if (LMO_FENCE_CTA) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
@@ -603,6 +609,11 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
 #if LMO_ATTN_PROFILE
             prof_gb = gtimer();
 #endif
+        }
+        __syncwarp();
+    };
+    auto prologue = [&](bool before_append) {   // (always called with true)
+        if (lane == 0) {
             int s = 0;
             for (; s < kStages && !ctl.pdone; ++s) {
                 if (before_append && a.k_new && holds_append_slot()) break;
@@ -742,14 +753,17 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
     // kernel has finished), then the wait, then q / new token.  Otherwise the small loads
     // go first.  Stages holding the append slot are held back until after the append.
     // (Stream-K / SM teams learn their first pair from the producer prologue.)
+    prologue_setup();
     if (early) {
         prologue(true);
         asm volatile("griddepcontrol.wait;\n" ::: "memory");
         fetch_first();
     } else if (!(TEAMK || wms.T)) {
+        if (!a.lens) asm volatile("griddepcontrol.wait;\n" ::: "memory");
         prologue(true);
         fetch_first();
     } else {
+        if (!a.lens) asm volatile("griddepcontrol.wait;\n" ::: "memory");
         fetch_first();
         prologue(true);
     }
@@ -807,6 +821,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
         }
         __syncwarp();
         const int seg_n = ctl.seg.sn, blk0 = ctl.seg.blk0, L = ctl.seg.L;
+        const int Lseg = min(L, (blk0 + seg_n) * kBlk);   // end (exclusive) of this segment's tokens
 #if LMO_ATTN_PROFILE
         ++prof_seg;
 #endif
@@ -856,9 +871,13 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
             prof_wait += clock64() - pw0;
 #endif
         };
-        // FULL: all kSub sub-blocks present and no ragged tail -> branch-free
+        // mode M (decltype(full)::value): 1 = FULL (all kSub sub-blocks present, no ragged
+        // tail: branch-free, no masking); 0 = GEN (sub-block count and tail tested);
+        // 2 = MASKED (LMO_UNIFIED: every sub-block computed, tokens >= Lseg masked -- one
+        // branch-free body for every stage of a segment, half the code)
         auto stage_k = [&](auto full, int sl, int jb, KState<D> &ks) {
-            constexpr bool F = decltype(full)::value;
+            constexpr int M = (int)decltype(full)::value;
+            constexpr bool F = M != 0;
             const uint32_t st = sl * GG::STAGE;
             const int nsub = F ? kSub : min(kSub, seg_n - jb);
             if constexpr (MHA) {
@@ -898,7 +917,8 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
                     z = fmaf(S[grp], f.y * zs24, fmaf(f.x * zs, qs[grp][0], z));
                 }
                 const int tokbase = (blk0 + jb + ls) * kBlk;
-                if (!F && (ls >= nsub || tokbase + row >= L)) z = NEG_INF;
+                if (M == 0 && (ls >= nsub || tokbase + row >= L)) z = NEG_INF;
+                if (M == 2 && tokbase + row >= Lseg) z = NEG_INF;
                 ks.z[0][0][0] = z;
             } else {
 #pragma unroll
@@ -938,9 +958,13 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
                         ks.z[s][r][1] = z1;
                     }
                     const int tokbase = (blk0 + jb + s) * kBlk;
-                    if (!F && tokbase + kBlk > L) {                 // ragged tail
+                    if (M == 0 && tokbase + kBlk > L) {                 // ragged tail
                         if (tokbase + tk0 >= L) ks.z[s][0][0] = ks.z[s][0][1] = NEG_INF;
                         if (tokbase + tk1 >= L) ks.z[s][1][0] = ks.z[s][1][1] = NEG_INF;
+                    }
+                    if (M == 2) {
+                        if (tokbase + tk0 >= Lseg) ks.z[s][0][0] = ks.z[s][0][1] = NEG_INF;
+                        if (tokbase + tk1 >= Lseg) ks.z[s][1][0] = ks.z[s][1][1] = NEG_INF;
                     }
                 } else {
                     ks.z[s][0][0] = ks.z[s][0][1] = ks.z[s][1][0] = ks.z[s][1][1] = NEG_INF;
@@ -951,10 +975,11 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
 
         // softmax + V part of one stage, then hand the slot back to the producer
         auto stage_v = [&](auto full, int sl, int jb, const KState<D> &ks) {
-            constexpr bool F = decltype(full)::value;
+            constexpr int M = (int)decltype(full)::value;
+            constexpr bool F = M != 0;
             const uint32_t st = sl * GG::STAGE;
             const int nsub = F ? kSub : min(kSub, seg_n - jb);
-            const bool tail = !F && (blk0 + jb + kSub) * kBlk > L;
+            const bool tail = M == 2 || (M == 0 && (blk0 + jb + kSub) * kBlk > L);
             if constexpr (MHA) {
                 // ---- one token per lane: warp-wide running max, p, V meta, w = p*scale
                 const int ls = t >> 1, hi = t & 1;
@@ -988,7 +1013,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
 #pragma unroll
                 for (int grp = 0; grp < NG; ++grp) {
                     float2 f = meta_f2(grp == 0 ? vmw.x : vmw.y);
-                    if (!F && z == NEG_INF) f = make_float2(0.f, 0.f);     // stale meta of masked slots
+                    if (M != 1 && z == NEG_INF) f = make_float2(0.f, 0.f);     // stale meta of masked slots
                     pm[0][grp] = fmaf(p, f.x, pm[0][grp]);
                     w[grp] = p * f.y;
                 }
@@ -1118,10 +1143,34 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
         // ragged tail take the branch-free FULL path (the hot loop); the rest
         // (at most the last one or two of a segment) take the general path.
         const int nst = (seg_n + kSub - 1) / kSub;
+        KState<D> kC, kN;
+        if constexpr (LMO_UNIFIED && MHA) {   // (measured: MHA gains, GQA loses)
+        const std::integral_constant<int, 2> MK{};
+        if (nst > 0) {
+            wait_stage(slot, phase);
+            stage_k(MK, slot, 0, kC);
+        }
+        int i = 0;
+#pragma unroll 1
+        for (; i + 1 < nst; ++i) {
+            int slN = slot;
+            uint32_t phN = phase;
+            advance(slN, phN);
+            wait_stage(slN, phN);
+            stage_k(MK, slN, (i + 1) * kSub, kN);
+            stage_v(MK, slot, i * kSub, kC);
+            slot = slN;
+            phase = phN;
+            kC = kN;
+        }
+        if (nst > 0) {            // the last stage's V part (peeled: keeps the loop body branch-free)
+            stage_v(MK, slot, i * kSub, kC);
+            advance(slot, phase);
+        }
+        } else {
         const int nfull = max(0, min(seg_n / kSub, (L / kBlk - blk0) / kSub));
         const std::true_type FULL{};
         const std::false_type GEN{};
-        KState<D> kC, kN;
         if (nst > 0) {
             wait_stage(slot, phase);
             if (nfull > 0) stage_k(FULL, slot, 0, kC);
@@ -1156,6 +1205,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
             slot = slN;
             phase = phN;
             kC = kN;
+        }
         }
 
         // ------------------------------------------------ segment end

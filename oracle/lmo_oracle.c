@@ -320,3 +320,36 @@ int lmo_oracle_decode_attention_q4(const uint8_t *k_codes, const uint16_t *k_met
     return lmo_oracle_decode_attention_q4_mt(k_codes, k_meta, v_codes, v_meta, B, Hkv, cap, d, q,
                                              Hq, lens, sigma, out, 1);
 }
+
+/* ------------------------------------------------- W4A16 linear (NEXT-3) */
+
+/* A linear layer over group-wise q4 weights: the paper quantizes the weights
+ * once and dequantizes them on the GPU each decode step before the layer's
+ * matmuls ("load_weight + dequan_wgt", Eq 4; "weights only cause
+ * de-quantization overhead on GPU" P:293-295; Eq 11).  The plain
+ * definition of that step is
+ *     y[b][n] = sum_k x[b][k] * W~[n][k],   W~ = D1 dequantization of W,
+ * with W quantized along k (groups of `group` consecutive input features of
+ * one output row: outer = N, n = K, inner = 1 in quantize_groupwise terms).
+ * Computed here in fp64 on the D1 fp16 values, k ascending.  x is fp16 bits
+ * [B][K]; codes [N][Kpad/2]; meta [N][Kpad/group][2]; y double [B][N]. */
+int lmo_oracle_w4a16_linear(const uint8_t *codes, const uint16_t *meta, int64_t N, int64_t K,
+                            int group, const uint16_t *x, int64_t B, double *y) {
+    if (N <= 0 || K <= 0 || B <= 0 || group <= 0 || group % 2 != 0) return LMO_ORACLE_EINVAL;
+    uint16_t *w = (uint16_t *)malloc((size_t)(N * K) * sizeof(uint16_t));
+    if (!w) return LMO_ORACLE_EINVAL;
+    int rc = lmo_oracle_dequantize_groupwise(codes, meta, N, K, 1, 4, group, w);   /* D1, Eq 11 */
+    if (rc) {
+        free(w);
+        return rc;
+    }
+    for (int64_t b = 0; b < B; ++b)
+        for (int64_t n = 0; n < N; ++n) {
+            double s = 0.0;
+            for (int64_t k = 0; k < K; ++k)
+                s += lmo_oracle_h2d(x[b * K + k]) * lmo_oracle_h2d(w[n * K + k]);
+            y[b * N + n] = s;
+        }
+    free(w);
+    return LMO_ORACLE_OK;
+}

@@ -19,7 +19,7 @@ CFLAGS = ["-O2", "-std=c11", "-fno-fast-math", "-ffp-contract=off", "-shared", "
           "-Wall", "-Wextra", "-pthread"]
 
 __all__ = ["build", "lib", "h2d", "rn16", "ru16", "quantize_groupwise", "dequantize_groupwise",
-           "kv_append_quant", "decode_attention_q4", "new_cache"]
+           "kv_append_quant", "decode_attention_q4", "new_cache", "w4a16_linear"]
 
 
 def build(force: bool = False) -> str:
@@ -52,7 +52,8 @@ def lib():
         L.lmo_oracle_kv_append_quant.argtypes = [P, P, P, P, i32, i32, i32, i32, P, P, i32, P]
         L.lmo_oracle_decode_attention_q4_mt.argtypes = [P, P, P, P, i32, i32, i32, i32, P, i32, P,
                                                         ctypes.c_double, P, i32]
-        for f in ("lmo_oracle_quantize_groupwise", "lmo_oracle_dequantize_groupwise",
+        L.lmo_oracle_w4a16_linear.argtypes = [P, P, i64, i64, i32, P, i64, P]
+        for f in ("lmo_oracle_quantize_groupwise", "lmo_oracle_dequantize_groupwise", "lmo_oracle_w4a16_linear",
                   "lmo_oracle_kv_append_quant", "lmo_oracle_decode_attention_q4_mt"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
@@ -164,3 +165,21 @@ def decode_attention_q4(cache: dict, q: np.ndarray, lens, sigma: float | None = 
     if rc:
         raise ValueError("oracle attention: invalid arguments")
     return out
+
+
+def w4a16_linear(codes: np.ndarray, meta: np.ndarray, N: int, K: int, x: np.ndarray,
+                 group: int = 64) -> np.ndarray:
+    """A linear layer over q4 weights (NEXT-3): y = x W~^T with W~ the Eq 11 / D1
+    dequantization of W [N][K] quantized along K -- the paper's per-step
+    "dequan_wgt" then matmul (Eq 4, P:228-233; P:293-295).  x fp16 [B][K];
+    returns float64 [B][N]."""
+    codes = np.ascontiguousarray(codes, dtype=np.uint8)
+    meta = np.ascontiguousarray(meta, dtype=np.uint16)
+    xb = _bits(x)
+    B = xb.size // K
+    assert xb.size == B * K
+    y = np.zeros((B, N), dtype=np.float64)
+    rc = lib().lmo_oracle_w4a16_linear(_ptr(codes), _ptr(meta), N, K, group, _ptr(xb), B, _ptr(y))
+    if rc:
+        raise ValueError("oracle w4a16: invalid arguments")
+    return y

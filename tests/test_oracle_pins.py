@@ -380,3 +380,81 @@ def test_attention_threads_identical():
     a = oracle.decode_attention_q4(cache, q, 33, nthreads=1)
     b = oracle.decode_attention_q4(cache, q, 33, nthreads=5)
     assert np.array_equal(a, b)
+
+
+# ------------------------------------------------------------ W4A16 (NEXT-3)
+def on_grid_matrix(rng, N, K, int_valued=True):
+    """W [N][K] whose every 64-group is on its own grid mn + k*step (k = 0..15,
+    both ends present), so Alg 2 + Eq 11 reproduce W exactly (pinned above)."""
+    W = np.zeros((N, K), np.float64)
+    for n in range(N):
+        for g in range(K // 64):
+            mn = float(rng.integers(-8, 8)) if int_valued else float(rng.integers(-64, 64)) / 8
+            step = float(rng.integers(1, 4)) if int_valued else float(rng.integers(1, 9)) / 16
+            k = rng.integers(0, 16, 64)
+            k[rng.choice(64, 2, replace=False)] = [0, 15]
+            W[n, g * 64:(g + 1) * 64] = mn + k * step
+    assert np.array_equal(W.astype(np.float16).astype(np.float64), W)
+    return W
+
+
+def test_w4a16_on_grid_integer_exact():
+    """y = x W^T (Eq 4's dequan_wgt then matmul) on integer-valued
+    x and on-grid integer W: every product and partial sum is an integer far
+    below 2^53, so the oracle must reproduce the exact integer matmul of the
+    ORIGINAL W -- a wrong code, group min/scale, k index or transpose fails."""
+    rng = np.random.default_rng(RNG_SEED + 40)
+    N, K, B = 7, 192, 5
+    W = on_grid_matrix(rng, N, K)
+    x = rng.integers(-20, 21, (B, K)).astype(np.float64)
+    c, m = oracle.quantize_groupwise(W.astype(np.float16), N, K, 1)
+    y = oracle.w4a16_linear(c, m, N, K, x.astype(np.float16))
+    want = np.array([[int(sum(int(x[b, k]) * int(W[n, k]) for k in range(K))) for n in range(N)]
+                     for b in range(B)], dtype=np.float64)
+    assert np.array_equal(y, want)
+
+
+def test_w4a16_unit_vectors_pick_dequantized_weights():
+    """x = e_k picks column k: y[k][n] = W~[n][k].  On-grid W (non-integer
+    steps) must come back exactly; off-grid W within the Eq 10/11 bound
+    |W - W~| <= scale/2 (+ the fp16 rounding of D1)."""
+    rng = np.random.default_rng(RNG_SEED + 41)
+    N, K = 6, 128
+    W = on_grid_matrix(rng, N, K, int_valued=False)
+    c, m = oracle.quantize_groupwise(W.astype(np.float16), N, K, 1)
+    y = oracle.w4a16_linear(c, m, N, K, np.eye(K, dtype=np.float16))
+    assert np.array_equal(y, W.T)
+    Wr = (rng.standard_normal((N, K)) * 0.05).astype(np.float16)
+    c, m = oracle.quantize_groupwise(Wr, N, K, 1)
+    y = oracle.w4a16_linear(c, m, N, K, np.eye(K, dtype=np.float16))
+    scale = np.array([[F(m[n, k // 64, 0, 1]) for k in range(K)] for n in range(N)], dtype=np.float64)
+    err = np.abs(y.T - Wr.astype(np.float64))
+    assert np.all(err <= scale / 2 * (1 + 2.0 ** -10) + 2.0 ** -24)
+
+
+def test_w4a16_constant_rows_and_padding():
+    """A constant row (scale 0, codes 0: reading 1) gives y = c * sum_k x.
+    K not a multiple of 64 is zero-padded at the end (Q0, pads take part in
+    min/max: reading 7): the result equals the explicitly padded problem."""
+    rng = np.random.default_rng(RNG_SEED + 42)
+    N, K, B = 3, 128, 4
+    W = np.zeros((N, K), np.float16)
+    W[0, :] = 1.5
+    W[1, :] = -0.25
+    W[2, :] = 3.0
+    x = rng.integers(-9, 10, (B, K)).astype(np.float16)
+    c, m = oracle.quantize_groupwise(W, N, K, 1)
+    y = oracle.w4a16_linear(c, m, N, K, x)
+    sx = x.astype(np.float64).sum(axis=1)
+    assert np.array_equal(y, np.outer(sx, [1.5, -0.25, 3.0]))
+    K2 = 100
+    W2 = (rng.standard_normal((N, K2)) * 0.1).astype(np.float16)
+    x2 = rng.standard_normal((B, K2)).astype(np.float16)
+    c2, m2 = oracle.quantize_groupwise(W2, N, K2, 1)
+    Wp = np.zeros((N, 128), np.float16)
+    Wp[:, :K2] = W2
+    xp = np.zeros((B, 128), np.float16)
+    xp[:, :K2] = x2
+    cp, mp = oracle.quantize_groupwise(Wp, N, 128, 1)
+    assert np.array_equal(c2, cp) and np.array_equal(m2, mp)
+    assert np.array_equal(oracle.w4a16_linear(c2, m2, N, K2, x2), oracle.w4a16_linear(cp, mp, N, 128, xp))

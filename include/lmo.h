@@ -240,6 +240,30 @@ lmo_status lmo_offload_decode_step(lmo_offload_t ex, const void *k_new_f16, cons
                                    void *compute_stream);
 lmo_status lmo_offload_destroy(lmo_offload_t ex);
 
+/* ---------------------------------------------------------------------------
+ * NEXT-3. Linear layer over group-wise q4 weights (W4A16), dequantization fused
+ * into the GEMM.  The paper dequantizes the q4 weights on the GPU every decode
+ * step before the layer's matmuls ("load_weight + dequan_wgt", Eq 4
+ * P:228-233; Eq 11); here the q4 codes stream from HBM
+ * and are expanded only in shared memory:
+ *     y[b][n] = sum_k x[b][k] * RN16(c[n][k] * scale[n][k/64] + min[n][k/64]).
+ *
+ * codes : W [N][K] quantized along K (lmo_quantize_groupwise with outer = N,
+ *         n = K, inner = 1): [N][K/2] bytes, low nibble = even k.
+ * meta  : [N][K/64] lmo_qmeta.
+ * x_f16 : activations [batch][K] fp16, row-major.
+ * y_f32 : output [batch][N] fp32, row-major (overwritten).
+ * N % 128 == 0, K % 64 == 0, 1 <= batch <= 128 (else LMO_ERR_SHAPE /
+ * LMO_ERR_UNSUPPORTED).  k_split: K-dimension split (0 = auto); with k_split
+ * > 1 y is zeroed on `stream` and the partial tiles are added atomically
+ * (summation order then varies: results agree within fp32 rounding).  All
+ * pointers 16-byte aligned.  Device memory is caller-owned; enqueued on
+ * `stream`, asynchronous.
+ * ------------------------------------------------------------------------- */
+lmo_status lmo_w4a16_linear(const uint8_t *codes, const lmo_qmeta *meta, int64_t N, int64_t K,
+                            const void *x_f16, int32_t batch, float *y_f32, int32_t k_split,
+                            void *stream);
+
 /* Human-readable name of a status code (static string). */
 const char *lmo_status_string(lmo_status status);
 

@@ -48,6 +48,8 @@ bool pdl_enabled() {
 cudaError_t launch_gen_fill(void *, int, int, int, int, uint64_t, int, int, int, int, int, int,
                             cudaStream_t);
 size_t attn_workspace_bytes(int B, int Hkv, int Hq, int D, int num_splits);
+cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const void *x, float *y, int N, int K,
+                         int batch, int ksplit, cudaStream_t st);
 
 static bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
@@ -202,6 +204,17 @@ size_t lmo_kv_row_bytes(int32_t head_dim) {
 }
 
 uint64_t lmo_launch_count(void) { return g_launches.load(std::memory_order_relaxed); }
+
+lmo_status lmo_w4a16_linear(const uint8_t *codes, const lmo_qmeta *meta, int64_t N, int64_t K,
+                            const void *x, int32_t batch, float *y, int32_t k_split, void *stream) {
+    if (!codes || !meta || !x || !y) return LMO_ERR_NULL;
+    if (N <= 0 || K <= 0 || batch <= 0 || k_split < 0) return LMO_ERR_SHAPE;
+    if (N % 128 != 0 || K % kGroup != 0 || N > (1ll << 30) || K > (1ll << 30)) return LMO_ERR_SHAPE;
+    if (batch > 128) return LMO_ERR_UNSUPPORTED;
+    if (!aligned16(codes) || !aligned16(meta) || !aligned16(x) || !aligned16(y)) return LMO_ERR_ALIGN;
+    return cuda_status(launch_w4a16(codes, meta, x, y, (int)N, (int)K, batch, k_split,
+                                    static_cast<cudaStream_t>(stream)));
+}
 
 uint32_t lmo_version(void) { return (1u << 16) | 0u; }
 

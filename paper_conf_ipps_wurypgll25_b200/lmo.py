@@ -49,6 +49,7 @@ def _load():
         "lmo_decode_attention_q4": [ctypes.POINTER(lmo_kv_cache), P, i32, i32, P, ctypes.c_float,
                                     i32, P, ctypes.c_int, P, ctypes.c_size_t, P],
         "lmo_gen_fill_f16": [P, i32, i32, i32, i32, u64, i32, i32, i32, i32, i32, i32, P],
+        "lmo_w4a16_linear": [P, P, i64, i64, P, i32, P, i32, P],
         "lmo_decode_step_q4": [ctypes.POINTER(lmo_kv_cache), P, P, P, i32, i32, P, ctypes.c_float,
                                i32, P, ctypes.c_int, P, ctypes.c_size_t, ctypes.c_uint32, P],
     }
@@ -86,7 +87,7 @@ EXPORTS = ["lmo_quantize_groupwise", "lmo_dequantize_groupwise", "lmo_kv_append_
            "lmo_status_string",
            "lmo_gen_fill_f16", "lmo_launch_count", "lmo_version",
            "lmo_offload_ring_bytes", "lmo_offload_create", "lmo_offload_decode_step",
-           "lmo_offload_destroy"]
+           "lmo_offload_destroy", "lmo_w4a16_linear"]
 
 
 def _check(status: int, fn: str) -> None:
@@ -142,6 +143,20 @@ def lmo_dequantize_groupwise(codes: torch.Tensor, meta: torch.Tensor, outer: int
     _check(_lib.lmo_dequantize_groupwise(_ptr(codes), _ptr(meta), outer, n, inner, bits,
                                          group_size, _ptr(y), _stream(stream)),
            "lmo_dequantize_groupwise")
+    return y
+
+
+def lmo_w4a16_linear(codes: torch.Tensor, meta: torch.Tensor, N: int, K: int, x: torch.Tensor,
+                     y: torch.Tensor | None = None, k_split: int = 0, stream=None) -> torch.Tensor:
+    """NEXT-3: y = x W~^T over q4 weights W [N][K] quantized along K (Eq 4's
+    load_weight + dequan_wgt then matmul), fused on the tensor cores.
+    x fp16 [batch][K]; returns fp32 [batch][N]."""
+    batch = x.numel() // K
+    if y is None:
+        y = torch.empty((batch, N), dtype=torch.float32, device=x.device)
+    _need_cuda(codes, meta, x, y)
+    _check(_lib.lmo_w4a16_linear(_ptr(codes), _ptr(meta), N, K, _ptr(x), batch, _ptr(y), k_split,
+                                 _stream(stream)), "lmo_w4a16_linear")
     return y
 
 

@@ -1,0 +1,130 @@
+"""GPU parity for NEXT-3, the W4A16 linear layer (tcgen05 GEMM with the
+dequantization fused in), through the C ABI, against the CPU oracle
+(oracle.w4a16_linear: fp64 matmul on the Eq 11 / D1 dequantized weights).
+
+Tolerance: the kernel dequantizes with one fp16 rounding
+RN16(c*scale + min) (HFMA2) where D1 rounds twice, RN16(RN32(.)) -- the two can
+differ by one fp16 ulp on double-rounding ties -- and accumulates in fp32 on
+the tensor cores.  Elementwise bar: |y - y_ref| <= 2^-10 * sum_k |x_k w_k|
++ 1e-6 (one ulp16 on every weight plus fp32 accumulation, far below the
+error of a wrong code, group or index, which is O(scale * |x|) per term).
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def lmo():
+    from paper_conf_ipps_wurypgll25_b200 import lmo as m
+    return m
+
+
+def make_weights(rng, N, K):
+    W = rng.standard_normal((N, K)) * 0.05
+    W[:, rng.choice(K, max(1, K // 50), replace=False)] *= 8.0      # outlier input features
+    W = W.astype(np.float16)
+    codes, meta = oracle.quantize_groupwise(W, N, K, 1)
+    return codes.reshape(N, K // 2), meta.reshape(N, K // 64, 2)
+
+
+def check(lmo, N, K, batch, k_split, seed):
+    rng = np.random.default_rng(seed)
+    codes, meta = make_weights(rng, N, K)
+    x = rng.standard_normal((batch, K)).astype(np.float16)
+    ref = oracle.w4a16_linear(codes, meta, N, K, x)
+    wdq = oracle.dequantize_groupwise(codes, meta, N, K, 1).reshape(N, K).astype(np.float64)
+    bound = np.abs(x.astype(np.float64)) @ np.abs(wdq).T * 2.0 ** -10 + 1e-6
+    y = lmo.lmo_w4a16_linear(torch.from_numpy(codes).cuda(), torch.from_numpy(meta.view(np.int32)).cuda(),
+                             N, K, torch.from_numpy(x).cuda(), k_split=k_split)
+    torch.cuda.synchronize()
+    got = y.cpu().numpy().astype(np.float64)
+    err = np.abs(got - ref)
+    assert np.all(err <= bound), (err.max(), (err / bound).max())
+    return got, ref
+
+
+@pytest.mark.parametrize("N,K,batch,k_split", [
+    (128, 64, 1, 1),          # one tile, one step
+    (256, 320, 5, 1),         # ragged batch (< 16), 5 groups
+    (256, 320, 5, 2),         # split-K, uneven
+    (384, 640, 64, 0),        # auto split
+    (128, 1024, 100, 3),      # BN = 128 instance, ragged batch
+    (256, 512, 128, 4),
+])
+def test_w4a16_vs_oracle(lmo, N, K, batch, k_split):
+    check(lmo, N, K, batch, k_split, seed=1000 + N + K + batch + k_split)
+
+
+def test_w4a16_split_invariant_and_deterministic(lmo):
+    """k_split = 1 is deterministic run to run; every split agrees with it
+    within fp32 rounding."""
+    rng = np.random.default_rng(7)
+    N, K, B = 256, 1024, 64
+    codes, meta = make_weights(rng, N, K)
+    x = torch.from_numpy(rng.standard_normal((B, K)).astype(np.float16)).cuda()
+    c, m = torch.from_numpy(codes).cuda(), torch.from_numpy(meta.view(np.int32)).cuda()
+    y1 = lmo.lmo_w4a16_linear(c, m, N, K, x, k_split=1).cpu()
+    y1b = lmo.lmo_w4a16_linear(c, m, N, K, x, k_split=1).cpu()
+    assert torch.equal(y1, y1b)
+    for s in (2, 4, 16):
+        ys = lmo.lmo_w4a16_linear(c, m, N, K, x, k_split=s).cpu()
+        assert torch.allclose(ys, y1, rtol=1e-5, atol=1e-4)
+
+
+def test_w4a16_on_grid_exact(lmo):
+    """On-grid integer weights and integer activations: every product and
+    partial sum is an integer < 2^24, so the tensor-core result is exact."""
+    rng = np.random.default_rng(11)
+    N, K, B = 128, 256, 16
+    W = np.zeros((N, K))
+    for n in range(N):
+        for g in range(K // 64):
+            k = rng.integers(0, 16, 64)
+            k[:2] = [0, 15]
+            W[n, g * 64:(g + 1) * 64] = float(rng.integers(-4, 4)) + k
+    x = rng.integers(-3, 4, (B, K)).astype(np.float16)
+    codes, meta = oracle.quantize_groupwise(W.astype(np.float16), N, K, 1)
+    y = lmo.lmo_w4a16_linear(torch.from_numpy(codes.reshape(N, K // 2)).cuda(),
+                             torch.from_numpy(meta.reshape(N, K // 64, 2).view(np.int32)).cuda(), N, K,
+                             torch.from_numpy(x).cuda(), k_split=1)
+    assert np.array_equal(y.cpu().numpy().astype(np.float64), x.astype(np.float64) @ W.T)
+
+
+def test_w4a16_config3_layer_sampled(lmo):
+    """OPT-30B (config 3) FFN1 shape at batch 64 -- N = 4*h1 = 28672, K = h1 =
+    7168 -- in the launch configuration the bench times (auto split); rows
+    sampled against the oracle."""
+    rng = np.random.default_rng(3)
+    N, K, B = 28672, 7168, 64
+    W = (rng.standard_normal((N, K), dtype=np.float32) * 0.02).astype(np.float16)
+    Wt = torch.from_numpy(W).cuda()
+    codes = torch.empty((N, K // 2), dtype=torch.uint8, device="cuda")
+    meta = torch.empty((N, K // 64), dtype=torch.int32, device="cuda")
+    lmo.lmo_quantize_groupwise(Wt, N, K, 1, codes=codes, meta=meta)
+    x = rng.standard_normal((B, K)).astype(np.float16)
+    y = lmo.lmo_w4a16_linear(codes, meta, N, K, torch.from_numpy(x).cuda()).cpu().numpy()
+    rows = np.sort(rng.choice(N, 24, replace=False))
+    ch = codes[rows].cpu().numpy()
+    mh = meta[rows].cpu().numpy().view(np.uint16).reshape(len(rows), K // 64, 2)
+    ref = oracle.w4a16_linear(ch, mh, len(rows), K, x)
+    wdq = oracle.dequantize_groupwise(ch, mh, len(rows), K, 1).reshape(len(rows), K).astype(np.float64)
+    bound = np.abs(x.astype(np.float64)) @ np.abs(wdq).T * 2.0 ** -10 + 1e-6
+    assert np.all(np.abs(y[:, rows] - ref) <= bound)
+
+
+def test_w4a16_argument_errors(lmo):
+    c = torch.zeros((128, 32), dtype=torch.uint8, device="cuda")
+    m = torch.zeros((128, 1), dtype=torch.int32, device="cuda")
+    x = torch.zeros((4, 64), dtype=torch.float16, device="cuda")
+    with pytest.raises(lmo.LmoError):
+        lmo.lmo_w4a16_linear(c, m, 100, 64, x)                     # N % 128
+    with pytest.raises(lmo.LmoError):
+        lmo.lmo_w4a16_linear(c, m, 128, 60, x[:, :60].contiguous())  # K % 64
+    xb = torch.zeros((129, 64), dtype=torch.float16, device="cuda")
+    with pytest.raises(lmo.LmoError):
+        lmo.lmo_w4a16_linear(c, m, 128, 64, xb)                    # batch > 128

@@ -15,16 +15,23 @@
 // {min, scale} fp16 pairs.  K % 64 == 0, N % 128 == 0.
 //
 // CTA tile: 128 output features (UMMA M) x BN batch columns (UMMA N), K in
-// 64-element steps (one quantization group = one 128-B swizzle atom):
-//   warps 0-7 (256 threads)  producers: cp.async of the raw codes / meta / x
-//                            kRaw steps ahead into a staging ring; dequant of
-//                            their row-half into the SWIZZLE_128B K-major A
-//                            stage; x copy into the B stage; then the epilogue
-//                            (warps 0-3: TMEM lanes = output rows)
-//   warp 8                   TMEM allocation, one elected lane issues
-//                            tcgen05.mma (4 x K=16 per step) and commits the
-//                            stage back to the producers.
+// 64-element steps (one quantization group):
+//   warp 9 (one lane)        TMA: the tile's q4 codes of step j (128 rows x 32 B,
+//                            2-D tensor map) into a kCodes-deep staging ring
+//   warp 10 (one lane)       TMA: the activations of step j (BN x 64 fp16, 2-D
+//                            tensor map, SWIZZLE_128B, rows >= batch zero-filled)
+//                            straight into the B operand stage
+//   warps 0-7 (256 threads)  dequant: thread (row r, half h) expands its 32
+//                            weights to fp16 and stores them with tcgen05.st
+//                            into the A operand stage in TENSOR MEMORY (lane =
+//                            row, 2 fp16 per column) -- the dequantized weights
+//                            never touch shared memory; then the epilogue
+//                            (warps 0-3: tcgen05.ld of the accumulator)
+//   warp 8                   TMEM allocation; one lane issues tcgen05.mma
+//                            (A from TMEM, B from smem; 4 x K=16 per step).
 // Split-K (grid.y) accumulates fp32 partial tiles with red.global.add.
+#include <cuda.h>
+
 #include "common.cuh"
 
 namespace lmo {
@@ -32,21 +39,33 @@ namespace lmo {
 namespace w4 {
 constexpr int kM = 128;          // output features per CTA (UMMA M)
 constexpr int kK = 64;           // K per stage (one group, one swizzle atom of fp16)
-constexpr int kStages = 3;       // A/B operand stages
-constexpr int kRaw = 4;          // cp.async staging depth (steps in flight)
-constexpr int kProd = 256;       // producer threads
-constexpr int kThreads = kProd + 32;
+#ifndef LMO_W4_STAGES
+#define LMO_W4_STAGES 4
+#endif
+#ifndef LMO_W4_CODES
+#define LMO_W4_CODES 12
+#endif
+constexpr int kStages = LMO_W4_STAGES;   // A (TMEM) / B (smem) operand stages
+constexpr int kCodes = LMO_W4_CODES;     // q4 code staging depth (steps in flight from HBM)
+constexpr int kProd = 256;               // dequant threads (warps 0-7)
+constexpr int kThreads = kProd + 96;     // + MMA warp, codes-TMA warp, x-TMA warp
 
 template <int BN>
 struct Smem {
-    static constexpr int A = kM * 128;                 // 16 KB
-    static constexpr int B = BN * 128;                 // BN x 64 fp16
-    static constexpr int STAGE = A + B;
-    static constexpr int RAW_CODES = kM * 32;          // 4 KB
-    static constexpr int RAW_META = kM * 8;          // one copy per row-half (thread-private)
-    static constexpr int RAW_X = BN * 128;
-    static constexpr int RAW = RAW_CODES + RAW_META + RAW_X;
-    static constexpr int BYTES = kStages * STAGE + kRaw * RAW + 1024 /* align */ + 256 /* barriers */;
+    static constexpr int B = BN * 128;                 // BN x 64 fp16, SWIZZLE_128B
+    static constexpr int CODES = kM * 32;              // 4 KB per step
+    static constexpr int META = kM * 8;                // per step: one 4-B copy per row-half (thread-private)
+    static constexpr int OFF_CODES = kStages * B;
+    static constexpr int OFF_META = OFF_CODES + kCodes * CODES;
+    static constexpr int OFF_BARS = OFF_META + kCodes * META;
+    static constexpr int BYTES = OFF_BARS + 256 + 1024 /* align */;
+};
+template <int BN>
+struct Tmem {
+    static constexpr int ACC = BN;                     // accumulator columns (fp32)
+    static constexpr int A0 = BN;                      // A stages: 32 columns each (64 fp16 per lane)
+    static constexpr int USED = BN + kStages * 32;
+    static constexpr int COLS = USED <= 32 ? 32 : USED <= 64 ? 64 : USED <= 128 ? 128 : USED <= 256 ? 256 : 512;
 };
 
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void *src, uint32_t src_bytes) {
@@ -99,38 +118,51 @@ __device__ __forceinline__ uint4 deq8(uint32_t w, __half2 sc, __half2 sc16, __ha
                       prmt(p2, p3, 0x7632u));
 }
 
+
+__device__ __forceinline__ void tma_2d(uint32_t dst, const void *tmap, int c0, int c1, uint64_t *bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n" ::"r"(dst),
+        "l"(tmap), "r"(c0), "r"(c1), "r"(smem_u32(bar))
+        : "memory");
+}
+
 template <int BN>
 __global__ void __launch_bounds__(kThreads, 1)
-w4a16_kernel(const uint8_t *__restrict__ codes, const uint32_t *__restrict__ meta,
-             const __half *__restrict__ x, float *__restrict__ y, int N, int K, int batch,
-             int ksplit) {
+w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant__ CUtensorMap tm_x,
+             const uint32_t *__restrict__ meta, float *__restrict__ y, int N, int K, int batch, int ksplit) {
     using S = Smem<BN>;
+    using TM = Tmem<BN>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint8_t *stages = smem;                                   // [kStages][A | B]
-    uint8_t *raw = smem + kStages * S::STAGE;                 // [kRaw][codes | meta | x]
-    uint64_t *bars = reinterpret_cast<uint64_t *>(raw + kRaw * S::RAW);
-    uint64_t *full = bars, *empty = bars + kStages, *done = bars + 2 * kStages;
-    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(bars + 2 * kStages + 1);
+    const uint32_t sbase = smem_u32(smem);
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + S::OFF_BARS);
+    uint64_t *c_full = bars, *c_empty = bars + kCodes;                    // codes ring
+    uint64_t *x_full = bars + 2 * kCodes, *a_full = x_full + kStages;     // operand stages
+    uint64_t *ab_empty = a_full + kStages, *done = ab_empty + kStages;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(done + 1);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int n0 = blockIdx.x * kM;
     const int KB = K / kK;
     const int kb0 = (int)((long long)blockIdx.y * KB / ksplit), kb1 = (int)((long long)(blockIdx.y + 1) * KB / ksplit);
     const int nsteps = kb1 - kb0;
-    constexpr int TCOLS = BN < 32 ? 32 : BN;                  // TMEM columns (power of 2 >= 32)
 
     if (tid == 0) {
+        for (int s = 0; s < kCodes; ++s) {
+            mbar_init(&c_full[s], 1);
+            mbar_init(&c_empty[s], kProd);
+        }
         for (int s = 0; s < kStages; ++s) {
-            mbar_init(&full[s], kProd);
-            mbar_init(&empty[s], 1);
+            mbar_init(&x_full[s], 1);
+            mbar_init(&a_full[s], kProd);
+            mbar_init(&ab_empty[s], 1);
         }
         mbar_init(done, 1);
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
-    if (warp == kProd / 32) {
+    if (warp == 8) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(smem_u32(tmem_slot)),
-                     "n"(TCOLS));
+                     "n"(TM::COLS));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n");
     }
     asm volatile("tcgen05.fence::before_thread_sync;\n");
@@ -138,80 +170,86 @@ w4a16_kernel(const uint8_t *__restrict__ codes, const uint32_t *__restrict__ met
     asm volatile("tcgen05.fence::after_thread_sync;\n");
     const uint32_t tmem = *tmem_slot;
 
-    if (tid < kProd) {
-        // ------------------------------------------------------------ producers
-        const int r = tid & (kM - 1), h = tid >> 7;             // row of the tile, half of the group
-        const uint8_t *crow = codes + (int64_t)(n0 + r) * (K / 2) + h * 16;
-        const uint32_t *mrow = meta + (int64_t)(n0 + r) * (K / kK);
-        const uint32_t raw_u32 = smem_u32(raw);
-        auto issue = [&](int j) {   // step j's raw data -> staging slot j % kRaw
-            if (j < nsteps) {
-                const int kb = kb0 + j;
-                const uint32_t base = raw_u32 + (j % kRaw) * S::RAW;
-                cp_async16(base + r * 32 + h * 16, crow + (int64_t)kb * 32, 16);
-                cp_async4(base + S::RAW_CODES + (h * kM + r) * 4, mrow + kb);
-                for (int c = tid; c < BN * 8; c += kProd) {       // x rows (zero beyond batch)
-                    const int xr = c >> 3, xc = c & 7;
-                    const bool ok = xr < batch;
-                    const __half *src = x + (int64_t)(ok ? xr : 0) * K + kb * kK + xc * 8;
-                    cp_async16(base + S::RAW_CODES + S::RAW_META + c * 16, src, ok ? 16 : 0);
-                }
+    if (warp == 9) {
+        // ------------------------------------------------------ TMA: q4 codes
+        if (lane == 0) {
+            for (int j = 0; j < nsteps; ++j) {
+                const int cs = j % kCodes;
+                if (j >= kCodes) mbar_wait(&c_empty[cs], ((j / kCodes) - 1) & 1);
+                mbar_arrive_expect_tx(&c_full[cs], S::CODES);
+                tma_2d(sbase + S::OFF_CODES + cs * S::CODES, &tm_codes, (kb0 + j) * 32, n0, &c_full[cs]);
             }
+        }
+    } else if (warp == 10) {
+        // ------------------------------------------------------ TMA: activations
+        if (lane == 0) {
+            for (int j = 0; j < nsteps; ++j) {
+                const int st = j % kStages;
+                if (j >= kStages) mbar_wait(&ab_empty[st], ((j / kStages) - 1) & 1);
+                mbar_arrive_expect_tx(&x_full[st], S::B);
+                tma_2d(sbase + st * S::B, &tm_x, (kb0 + j) * kK, 0, &x_full[st]);
+            }
+        }
+    } else if (warp < 8) {
+        // ------------------------------------------------------ dequant -> TMEM
+        const int r = tid & (kM - 1), h = tid >> 7;             // TMEM lane r (warp % 4 quarter), half h
+        const uint32_t *mrow = meta + (int64_t)(n0 + r) * (K / kK);
+        const uint32_t meta_u32 = sbase + S::OFF_META + (h * kM + r) * 4;
+        auto meta_issue = [&](int j) {   // thread-private cp.async ring of the group meta words
+            if (j < nsteps) cp_async4(meta_u32 + (j % kCodes) * S::META, mrow + kb0 + j);
             cp_commit();
         };
-        for (int j = 0; j < kRaw - 1; ++j) issue(j);
+        for (int j = 0; j < kCodes - 1; ++j) meta_issue(j);
+        const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16) + TM::A0 + h * 16;
         for (int j = 0; j < nsteps; ++j) {
-            issue(j + kRaw - 1);
-            cp_wait<kRaw - 1>();                                 // this thread's copies of step j
-            const int st = j % kStages;
-            if (j >= kStages) mbar_wait(&empty[st], ((j / kStages) - 1) & 1);
-            const uint8_t *rs = raw + (j % kRaw) * S::RAW;
-            uint8_t *A = stages + st * S::STAGE;
-            uint8_t *Bs = A + S::A;
-            // dequantize this thread's 32 weights (row r, k = 32h .. 32h+31)
-            const uint4 cw = *reinterpret_cast<const uint4 *>(rs + r * 32 + h * 16);
-            const uint32_t mw = *reinterpret_cast<const uint32_t *>(rs + S::RAW_CODES + (h * kM + r) * 4);
-            const __half mnh = __ushort_as_half((unsigned short)(mw & 0xFFFFu));
-            const __half sch = __ushort_as_half((unsigned short)(mw >> 16));
-            const __half2 mn2 = __half2half2(mnh), sc2 = __half2half2(sch);
-            const __half2 sc16 = __hmul2(sc2, __half2half2(__float2half_rn(0.0625f)));
-            const uint32_t words[4] = {cw.x, cw.y, cw.z, cw.w};
-#pragma unroll
-            for (int i = 0; i < 4; ++i) {
-                const uint4 v = deq8(words[i], sc2, sc16, mn2);
-                const int chunk = (h * 4 + i) ^ (r & 7);                 // SWIZZLE_128B
-                *reinterpret_cast<uint4 *>(A + r * 128 + chunk * 16) = v;
-            }
-            // activations: raw [BN][8 chunks] -> swizzled B stage
-            for (int c = tid; c < BN * 8; c += kProd) {
-                const int xr = c >> 3, xc = c & 7;
-                const uint4 v = *reinterpret_cast<const uint4 *>(rs + S::RAW_CODES + S::RAW_META + c * 16);
-                *reinterpret_cast<uint4 *>(Bs + xr * 128 + ((xc ^ (xr & 7)) * 16)) = v;
-            }
-            asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-            mbar_arrive(&full[st]);
+            meta_issue(j + kCodes - 1);
+            const int cs = j % kCodes, st = j % kStages;
+            mbar_wait(&c_full[cs], (j / kCodes) & 1);
+            uint32_t c0, c1, c2, c3, mw;
+            asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
+                         : "=r"(c0), "=r"(c1), "=r"(c2), "=r"(c3)
+                         : "r"(sbase + S::OFF_CODES + cs * S::CODES + r * 32 + h * 16));
+            mbar_arrive(&c_empty[cs]);
+            cp_wait<kCodes - 1>();
+            asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(meta_u32 + cs * S::META));
+            const __half2 mn2 = __half2half2(__ushort_as_half((unsigned short)(mw & 0xFFFFu)));
+            const __half2 sc2 = __half2half2(__ushort_as_half((unsigned short)(mw >> 16)));
+            const __half2 sc16 = __hmul2(sc2, __half2half2(__ushort_as_half(0x2C00)));   // * 1/16
+            const uint4 v0 = deq8(c0, sc2, sc16, mn2), v1 = deq8(c1, sc2, sc16, mn2);
+            const uint4 v2 = deq8(c2, sc2, sc16, mn2), v3 = deq8(c3, sc2, sc16, mn2);
+            if (j >= kStages) mbar_wait(&ab_empty[st], ((j / kStages) - 1) & 1);
+            asm volatile("tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};\n" ::"r"(
+                             lane_base + st * 32),
+                         "r"(v0.x), "r"(v0.y), "r"(v0.z), "r"(v0.w), "r"(v1.x), "r"(v1.y), "r"(v1.z), "r"(v1.w), "r"(v2.x),
+                         "r"(v2.y), "r"(v2.z), "r"(v2.w), "r"(v3.x), "r"(v3.y), "r"(v3.z), "r"(v3.w)
+                         : "memory");
+            asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
+            asm volatile("tcgen05.fence::before_thread_sync;\n");
+            mbar_arrive(&a_full[st]);
         }
         cp_wait<0>();
     } else {
-        // ------------------------------------------------------------ MMA issuer
+        // ------------------------------------------------------ MMA issuer (warp 8)
         constexpr uint32_t idesc = umma_idesc<BN>();
         for (int j = 0; j < nsteps; ++j) {
             const int st = j % kStages;
-            mbar_wait(&full[st], (j / kStages) & 1);
+            mbar_wait(&x_full[st], (j / kStages) & 1);
+            mbar_wait(&a_full[st], (j / kStages) & 1);
             asm volatile("tcgen05.fence::after_thread_sync;\n");
             if (lane == 0) {
-                const uint32_t a0 = smem_u32(stages + st * S::STAGE), b0 = a0 + S::A;
+                const uint32_t b0 = sbase + st * S::B;
 #pragma unroll
                 for (int k = 0; k < kK / 16; ++k) {
-                    const uint64_t da = umma_desc(a0 + k * 32), db = umma_desc(b0 + k * 32);
+                    const uint32_t ta = tmem + TM::A0 + st * 32 + k * 8;
+                    const uint64_t db = umma_desc(b0 + k * 32);
                     const uint32_t acc = (j > 0 || k > 0) ? 1u : 0u;
                     asm volatile(
                         "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-                        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem),
-                        "l"(da), "l"(db), "r"(idesc), "r"(acc));
+                        "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem),
+                        "r"(ta), "l"(db), "r"(idesc), "r"(acc));
                 }
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
-                                 smem_u32(&empty[st]))
+                                 smem_u32(&ab_empty[st]))
                              : "memory");
             }
             __syncwarp();
@@ -259,9 +297,9 @@ w4a16_kernel(const uint8_t *__restrict__ codes, const uint32_t *__restrict__ met
     }
     asm volatile("tcgen05.fence::before_thread_sync;\n");
     __syncthreads();
-    if (warp == kProd / 32) {
+    if (warp == 8) {
         asm volatile("tcgen05.fence::after_thread_sync;\n");
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "n"(TCOLS));
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "n"(TM::COLS));
     }
 }
 
@@ -275,28 +313,63 @@ int w4a16_auto_split(int N, int K) {
     return s;
 }
 
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
+                                  const cuuint64_t *, const cuuint32_t *, const cuuint32_t *, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+static EncodeTiledFn encode_tiled() {
+    static EncodeTiledFn fn = nullptr;
+    if (!fn) {
+        void *p = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            fn = reinterpret_cast<EncodeTiledFn>(p);
+    }
+    return fn;
+}
+
 cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const void *x, float *y, int N, int K,
                          int batch, int ksplit, cudaStream_t st) {
     if (ksplit <= 0) ksplit = w4a16_auto_split(N, K);
     if (ksplit > K / w4::kK) ksplit = K / w4::kK;
+    EncodeTiledFn enc = encode_tiled();
+    if (!enc) return cudaErrorNotSupported;
+    const int BN = batch <= 64 ? 64 : 128;
+    CUtensorMap tc, tx;
+    {   // codes [N][K/2] u8, box 32 B x 128 rows
+        const cuuint64_t dims[2] = {(cuuint64_t)K / 2, (cuuint64_t)N};
+        const cuuint64_t strides[1] = {(cuuint64_t)K / 2};
+        const cuuint32_t box[2] = {32, (cuuint32_t)w4::kM}, es[2] = {1, 1};
+        if (enc(&tc, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t *>(codes), dims, strides, box, es,
+                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+            return cudaErrorInvalidValue;
+    }
+    {   // x [batch][K] fp16, box 64 x BN rows, SWIZZLE_128B (rows >= batch are zero-filled)
+        const cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)batch};
+        const cuuint64_t strides[1] = {(cuuint64_t)K * 2};
+        const cuuint32_t box[2] = {(cuuint32_t)w4::kK, (cuuint32_t)BN}, es[2] = {1, 1};
+        if (enc(&tx, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void *>(x), dims, strides, box, es,
+                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+            return cudaErrorInvalidValue;
+    }
     if (ksplit > 1) {
         const cudaError_t e = cudaMemsetAsync(y, 0, (size_t)batch * N * sizeof(float), st);
         if (e != cudaSuccess) return e;
     }
     dim3 grid(N / w4::kM, ksplit);
-    cudaError_t e;
-    if (batch <= 64) {
+    const uint32_t *m = static_cast<const uint32_t *>(meta);
+    if (BN == 64) {
         const int sm = w4::Smem<64>::BYTES;
         cudaFuncSetAttribute(w4::w4a16_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
-        w4::w4a16_kernel<64><<<grid, w4::kThreads, sm, st>>>(codes, static_cast<const uint32_t *>(meta),
-                                                              static_cast<const __half *>(x), y, N, K, batch, ksplit);
+        w4::w4a16_kernel<64><<<grid, w4::kThreads, sm, st>>>(tc, tx, m, y, N, K, batch, ksplit);
     } else {
         const int sm = w4::Smem<128>::BYTES;
         cudaFuncSetAttribute(w4::w4a16_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
-        w4::w4a16_kernel<128><<<grid, w4::kThreads, sm, st>>>(codes, static_cast<const uint32_t *>(meta),
-                                                               static_cast<const __half *>(x), y, N, K, batch, ksplit);
+        w4::w4a16_kernel<128><<<grid, w4::kThreads, sm, st>>>(tc, tx, m, y, N, K, batch, ksplit);
     }
-    e = cudaGetLastError();
+    const cudaError_t e = cudaGetLastError();
     if (e == cudaSuccess) note_launch();
     return e;
 }

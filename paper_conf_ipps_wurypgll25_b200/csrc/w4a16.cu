@@ -16,6 +16,8 @@
 //
 // CTA tile: 128 output features (UMMA M) x BN batch columns (UMMA N), K in
 // 64-element steps (one quantization group):
+//   (warp ids below for LMO_W4_PARTS = 2; the default, 1 thread per weight row, uses
+//   dequant warps 0-3, MMA warp 4, TMA warps 5 and 6 -- measured best)
 //   warp 9 (one lane)        TMA: the tile's q4 codes of step j (128 rows x 32 B,
 //                            2-D tensor map) into a kCodes-deep staging ring
 //   warp 10 (one lane)       TMA: the activations of step j (BN x 64 fp16, 2-D
@@ -47,14 +49,20 @@ constexpr int kK = 64;           // K per stage (one group, one swizzle atom of 
 #endif
 constexpr int kStages = LMO_W4_STAGES;   // A (TMEM) / B (smem) operand stages
 constexpr int kCodes = LMO_W4_CODES;     // q4 code staging depth (steps in flight from HBM)
-constexpr int kProd = 256;               // dequant threads (warps 0-7)
-constexpr int kThreads = kProd + 96;     // + MMA warp, codes-TMA warp, x-TMA warp
+#ifndef LMO_W4_PARTS
+#define LMO_W4_PARTS 1
+#endif
+constexpr int kParts = LMO_W4_PARTS;     // dequant threads per weight row (each: 64/kParts weights per step)
+constexpr int kProd = 128 * kParts;      // dequant threads
+constexpr int kWMMA = kProd / 32;        // warp ids: MMA issuer, codes TMA, activation TMA
+constexpr int kWTC = kWMMA + 1, kWTX = kWMMA + 2;
+constexpr int kThreads = kProd + 96;
 
 template <int BN>
 struct Smem {
     static constexpr int B = BN * 128;                 // BN x 64 fp16, SWIZZLE_128B
     static constexpr int CODES = kM * 32;              // 4 KB per step
-    static constexpr int META = kM * 8;                // per step: one 4-B copy per row-half (thread-private)
+    static constexpr int META = kM * 4 * kParts;       // per step: one 4-B copy per thread (thread-private)
     static constexpr int OFF_CODES = kStages * B;
     static constexpr int OFF_META = OFF_CODES + kCodes * CODES;
     static constexpr int OFF_BARS = OFF_META + kCodes * META;
@@ -160,7 +168,7 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
         mbar_init(done, 1);
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
-    if (warp == 8) {
+    if (warp == kWMMA) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(smem_u32(tmem_slot)),
                      "n"(TM::COLS));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n");
@@ -170,7 +178,7 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
     asm volatile("tcgen05.fence::after_thread_sync;\n");
     const uint32_t tmem = *tmem_slot;
 
-    if (warp == 9) {
+    if (warp == kWTC) {
         // ------------------------------------------------------ TMA: q4 codes
         if (lane == 0) {
             for (int j = 0; j < nsteps; ++j) {
@@ -180,7 +188,7 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                 tma_2d(sbase + S::OFF_CODES + cs * S::CODES, &tm_codes, (kb0 + j) * 32, n0, &c_full[cs]);
             }
         }
-    } else if (warp == 10) {
+    } else if (warp == kWTX) {
         // ------------------------------------------------------ TMA: activations
         if (lane == 0) {
             for (int j = 0; j < nsteps; ++j) {
@@ -190,9 +198,10 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                 tma_2d(sbase + st * S::B, &tm_x, (kb0 + j) * kK, 0, &x_full[st]);
             }
         }
-    } else if (warp < 8) {
+    } else if (warp < kWMMA) {
         // ------------------------------------------------------ dequant -> TMEM
-        const int r = tid & (kM - 1), h = tid >> 7;             // TMEM lane r (warp % 4 quarter), half h
+        constexpr int WPT = kK / kParts;                        // weights per thread per step
+        const int r = tid & (kM - 1), h = tid >> 7;             // TMEM lane r (warp % 4 quarter), part h
         const uint32_t *mrow = meta + (int64_t)(n0 + r) * (K / kK);
         const uint32_t meta_u32 = sbase + S::OFF_META + (h * kM + r) * 4;
         auto meta_issue = [&](int j) {   // thread-private cp.async ring of the group meta words
@@ -200,29 +209,59 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
             cp_commit();
         };
         for (int j = 0; j < kCodes - 1; ++j) meta_issue(j);
-        const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16) + TM::A0 + h * 16;
+        const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16) + TM::A0 + h * (WPT / 2);
         for (int j = 0; j < nsteps; ++j) {
             meta_issue(j + kCodes - 1);
             const int cs = j % kCodes, st = j % kStages;
             mbar_wait(&c_full[cs], (j / kCodes) & 1);
-            uint32_t c0, c1, c2, c3, mw;
-            asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
-                         : "=r"(c0), "=r"(c1), "=r"(c2), "=r"(c3)
-                         : "r"(sbase + S::OFF_CODES + cs * S::CODES + r * 32 + h * 16));
+            uint32_t cw[WPT / 8], mw;
+            const uint32_t caddr = sbase + S::OFF_CODES + cs * S::CODES + r * 32 + h * (WPT / 2);
+            if constexpr (WPT == 64) {
+                asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
+                             : "=r"(cw[0]), "=r"(cw[1]), "=r"(cw[2]), "=r"(cw[3]) : "r"(caddr));
+                asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
+                             : "=r"(cw[4]), "=r"(cw[5]), "=r"(cw[6]), "=r"(cw[7]) : "r"(caddr + 16));
+            } else if constexpr (WPT == 32)
+                asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
+                             : "=r"(cw[0]), "=r"(cw[1]), "=r"(cw[2]), "=r"(cw[3]) : "r"(caddr));
+            else
+                asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n" : "=r"(cw[0]), "=r"(cw[1]) : "r"(caddr));
             mbar_arrive(&c_empty[cs]);
             cp_wait<kCodes - 1>();
             asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(meta_u32 + cs * S::META));
             const __half2 mn2 = __half2half2(__ushort_as_half((unsigned short)(mw & 0xFFFFu)));
             const __half2 sc2 = __half2half2(__ushort_as_half((unsigned short)(mw >> 16)));
             const __half2 sc16 = __hmul2(sc2, __half2half2(__ushort_as_half(0x2C00)));   // * 1/16
-            const uint4 v0 = deq8(c0, sc2, sc16, mn2), v1 = deq8(c1, sc2, sc16, mn2);
-            const uint4 v2 = deq8(c2, sc2, sc16, mn2), v3 = deq8(c3, sc2, sc16, mn2);
+            uint4 v[WPT / 8];
+#pragma unroll
+            for (int i = 0; i < WPT / 8; ++i) v[i] = deq8(cw[i], sc2, sc16, mn2);
             if (j >= kStages) mbar_wait(&ab_empty[st], ((j / kStages) - 1) & 1);
-            asm volatile("tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};\n" ::"r"(
-                             lane_base + st * 32),
-                         "r"(v0.x), "r"(v0.y), "r"(v0.z), "r"(v0.w), "r"(v1.x), "r"(v1.y), "r"(v1.z), "r"(v1.w), "r"(v2.x),
-                         "r"(v2.y), "r"(v2.z), "r"(v2.w), "r"(v3.x), "r"(v3.y), "r"(v3.z), "r"(v3.w)
-                         : "memory");
+            if constexpr (WPT == 64)
+                asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+                             "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};\n" ::"r"(lane_base + st * 32),
+                             "r"(v[0].x), "r"(v[0].y), "r"(v[0].z), "r"(v[0].w), "r"(v[1].x), "r"(v[1].y), "r"(v[1].z),
+                             "r"(v[1].w), "r"(v[2 % (WPT / 8)].x), "r"(v[2 % (WPT / 8)].y), "r"(v[2 % (WPT / 8)].z),
+                             "r"(v[2 % (WPT / 8)].w), "r"(v[3 % (WPT / 8)].x), "r"(v[3 % (WPT / 8)].y),
+                             "r"(v[3 % (WPT / 8)].z), "r"(v[3 % (WPT / 8)].w), "r"(v[4 % (WPT / 8)].x),
+                             "r"(v[4 % (WPT / 8)].y), "r"(v[4 % (WPT / 8)].z), "r"(v[4 % (WPT / 8)].w),
+                             "r"(v[5 % (WPT / 8)].x), "r"(v[5 % (WPT / 8)].y), "r"(v[5 % (WPT / 8)].z),
+                             "r"(v[5 % (WPT / 8)].w), "r"(v[6 % (WPT / 8)].x), "r"(v[6 % (WPT / 8)].y),
+                             "r"(v[6 % (WPT / 8)].z), "r"(v[6 % (WPT / 8)].w), "r"(v[7 % (WPT / 8)].x),
+                             "r"(v[7 % (WPT / 8)].y), "r"(v[7 % (WPT / 8)].z), "r"(v[7 % (WPT / 8)].w)
+                             : "memory");
+            else if constexpr (WPT == 32)
+                asm volatile("tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};\n" ::"r"(
+                                 lane_base + st * 32),
+                             "r"(v[0].x), "r"(v[0].y), "r"(v[0].z), "r"(v[0].w), "r"(v[1].x), "r"(v[1].y), "r"(v[1].z),
+                             "r"(v[1].w), "r"(v[WPT / 8 - 2].x), "r"(v[WPT / 8 - 2].y), "r"(v[WPT / 8 - 2].z),
+                             "r"(v[WPT / 8 - 2].w), "r"(v[WPT / 8 - 1].x), "r"(v[WPT / 8 - 1].y), "r"(v[WPT / 8 - 1].z),
+                             "r"(v[WPT / 8 - 1].w)
+                             : "memory");
+            else
+                asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};\n" ::"r"(lane_base + st * 32),
+                             "r"(v[0].x), "r"(v[0].y), "r"(v[0].z), "r"(v[0].w), "r"(v[WPT / 8 - 1].x),
+                             "r"(v[WPT / 8 - 1].y), "r"(v[WPT / 8 - 1].z), "r"(v[WPT / 8 - 1].w)
+                             : "memory");
             asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
             asm volatile("tcgen05.fence::before_thread_sync;\n");
             mbar_arrive(&a_full[st]);
@@ -297,7 +336,7 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
     }
     asm volatile("tcgen05.fence::before_thread_sync;\n");
     __syncthreads();
-    if (warp == 8) {
+    if (warp == kWMMA) {
         asm volatile("tcgen05.fence::after_thread_sync;\n");
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "n"(TM::COLS));
     }

@@ -398,6 +398,58 @@ def run_ours(args):
                          "peak": peak, **res}
             del xw, codes, meta, yw
 
+    # ---- NEXT-3 leg: one layer's linear layers over q4 weights (QKV 3h x h, O h x h,
+    # FFN1 4h x h, FFN2 h x 4h: the paper's 4 h1^2 + 2 h1 h2) at this GPU's
+    # batch through lmo_w4a16_linear (dequantization fused into the tcgen05 GEMM), vs the
+    # paper's path -- dequantize (A5) then an fp16 cuBLAS matmul (Eq 4).
+    w4a16 = None
+    if not args.no_stream and w.hidden > 0 and B <= 128:
+        h = w.hidden
+        shapes = [("qkv", 3 * h, h), ("o", h, h), ("ffn1", 4 * h, h), ("ffn2", h, 4 * h)]
+        with torch.cuda.stream(stream):
+            gen = torch.Generator(device=dev)
+            gen.manual_seed(seed + 1)
+            mats = []
+            for name, N_, K_ in shapes:
+                wt = (torch.randn((N_, K_), generator=gen, device=dev) * 0.02).half()
+                c_, m_ = lmo.lmo_quantize_groupwise(wt, N_, K_, 1, stream=stream)
+                xa = torch.randn((B, K_), generator=gen, device=dev).half()
+                mats.append((name, N_, K_, c_.view(N_, K_ // 2), m_.view(N_, K_ // 64), xa,
+                             torch.empty((B, N_), device=dev)))
+                del wt
+            wd = torch.empty((max(N_ * K_ for _, N_, K_ in shapes),), dtype=torch.float16, device=dev)
+
+            def fused():
+                for _, N_, K_, c_, m_, xa, ya in mats:
+                    lmo.lmo_w4a16_linear(c_, m_, N_, K_, xa, y=ya, stream=stream)
+
+            def dq_cublas():
+                for _, N_, K_, c_, m_, xa, ya in mats:
+                    wv = wd[:N_ * K_].view(N_, K_)
+                    lmo.lmo_dequantize_groupwise(c_, m_, N_, K_, 1, y=wv.view(N_, K_, 1), stream=stream)
+                    torch.matmul(xa, wv.t())
+
+            def timeit(fn, reps=10):
+                fn()
+                q0, q1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                q0.record(stream)
+                for _ in range(reps):
+                    fn()
+                q1.record(stream)
+                q1.synchronize()
+                return reduce_max(q0.elapsed_time(q1)) / reps
+
+            t_f, t_b = timeit(fused), timeit(dq_cublas)
+            by = sum(N_ * K_ * 0.5625 + B * K_ * 2 + B * N_ * 4 for _, N_, K_ in shapes)
+            fl = sum(2.0 * B * N_ * K_ for _, N_, K_ in shapes)
+            w4a16 = {"kernel": "w4a16_kernel (lmo_w4a16_linear; tcgen05, A = dequantized weights in TMEM)",
+                     "shapes": {n_: [N_, K_] for n_, N_, K_ in shapes}, "batch": B,
+                     "us_per_layer": t_f * 1e3, "GB/s": by / (t_f / 1e3) / 1e9,
+                     "frac": by / (t_f / 1e3) / 1e9 / peak, "TFLOP/s": fl / (t_f / 1e3) / 1e12,
+                     "algorithmic_bytes": by,
+                     "dequant_then_cublas_us_per_layer": t_b * 1e3, "speedup_vs_dequant_then_cublas": t_b / t_f}
+            del mats, wd
+
     # ---- NEXT-4 leg: the same decode step with every layer's q4 cache offloaded to pinned
     # host memory (the paper's setting, Alg 1): per layer a strided H2D of the old rows
     # into a 3-slot device ring, the fused step, a D2H of the new row (lmo_offload_*).
@@ -530,6 +582,7 @@ def run_ours(args):
                          "per_launch_us": attn_ms * 1e3, "algorithmic_bytes_per_launch": attn_bytes},
             "prefill_ms_all_layers": pre_ms,
             "streaming": streaming,
+            "w4a16": w4a16,
             "offload": offload,
             "gpu_launches": launches_per_step * args.steps,
             "clocks": clocks,

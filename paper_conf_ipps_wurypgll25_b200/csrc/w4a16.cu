@@ -49,6 +49,9 @@ constexpr int kK = 64;           // K per stage (one group, one swizzle atom of 
 #endif
 constexpr int kStages = LMO_W4_STAGES;   // A (TMEM) / B (smem) operand stages
 constexpr int kCodes = LMO_W4_CODES;     // q4 code staging depth (steps in flight from HBM)
+#ifndef LMO_W4_NODEQ
+#define LMO_W4_NODEQ 0
+#endif
 #ifndef LMO_W4_PARTS
 #define LMO_W4_PARTS 1
 #endif
@@ -234,7 +237,13 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
             const __half2 sc16 = __hmul2(sc2, __half2half2(__ushort_as_half(0x2C00)));   // * 1/16
             uint4 v[WPT / 8];
 #pragma unroll
-            for (int i = 0; i < WPT / 8; ++i) v[i] = deq8(cw[i], sc2, sc16, mn2);
+            for (int i = 0; i < WPT / 8; ++i) {
+#if LMO_W4_NODEQ   // (experiment: pipeline / MMA bound without the dequant arithmetic)
+                v[i] = make_uint4(cw[i], cw[i] ^ mw, cw[i], cw[i]);
+#else
+                v[i] = deq8(cw[i], sc2, sc16, mn2);
+#endif
+            }
             if (j >= kStages) mbar_wait(&ab_empty[st], ((j / kStages) - 1) & 1);
             if constexpr (WPT == 64)
                 asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"

@@ -59,6 +59,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_UNIFIED
 #define LMO_UNIFIED 1    // MHA: one masked loop body for every stage (0: separate FULL / GEN bodies)
 #endif
+#ifndef LMO_GQA_VOTE
+#define LMO_GQA_VOTE 0   // GQA FULL stages: rescale only when a running max moved (one vote)
+#endif
 #ifndef LMO_NO_SCH
 #define LMO_NO_SCH 0     // 1: every schedule runs the generic kernel instance (experiments)
 #endif
@@ -1062,7 +1065,7 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
             const float mn0 = fmaxf(m_run[0], mb0), mn1 = fmaxf(m_run[1], mb1);
             // (non-lazy builds: FULL stages rescale unconditionally, branch-free; GEN stages
             // skip it when no running max moved)
-            if (LMO_LAZY_MAX || F || __any_sync(0xffffffffu, (mn0 > m_run[0]) || (mn1 > m_run[1]))) {
+            if (LMO_LAZY_MAX || (F && !LMO_GQA_VOTE) || __any_sync(0xffffffffu, (mn0 > m_run[0]) || (mn1 > m_run[1]))) {
                 const float a0 = fast_exp2(m_run[0] - mn0), a1 = fast_exp2(m_run[1] - mn1);
                 m_run[0] = mn0;
                 m_run[1] = mn1;

@@ -60,7 +60,7 @@ constexpr int kStageTok = kBlk * kSub;
 #define LMO_UNIFIED 1    // MHA: one masked loop body for every stage (0: separate FULL / GEN bodies)
 #endif
 #ifndef LMO_GQA_VOTE
-#define LMO_GQA_VOTE 0   // GQA FULL stages: rescale only when a running max moved (one vote)
+#define LMO_GQA_VOTE 1   // GQA FULL stages: rescale only when a running max moved (one vote)
 #endif
 #ifndef LMO_NO_SCH
 #define LMO_NO_SCH 0     // 1: every schedule runs the generic kernel instance (experiments)

@@ -49,6 +49,15 @@ constexpr int kK = 64;           // K per stage (one group, one swizzle atom of 
 #endif
 constexpr int kStages = LMO_W4_STAGES;   // A (TMEM) / B (smem) operand stages
 constexpr int kCodes = LMO_W4_CODES;     // q4 code staging depth (steps in flight from HBM)
+#ifndef LMO_W4_XSTAGES
+#define LMO_W4_XSTAGES 4
+#endif
+constexpr int kX = LMO_W4_XSTAGES;       // B (activation) stages in smem: prefetched further ahead than A
+#ifndef LMO_W4_CPS
+#define LMO_W4_CPS 1
+#endif
+constexpr int kCPS = LMO_W4_CPS;         // steps per codes TMA (box 32*kCPS B x 128 rows: full lines)
+constexpr int kCodeSlots = kCodes / kCPS;
 #ifndef LMO_W4_NODEQ
 #define LMO_W4_NODEQ 0
 #endif
@@ -66,11 +75,13 @@ struct Smem {
     static constexpr int B = BN * 128;                 // BN x 64 fp16, SWIZZLE_128B
     static constexpr int CODES = kM * 32;              // 4 KB per step
     static constexpr int META = kM * 4 * kParts;       // per step: one 4-B copy per thread (thread-private)
-    static constexpr int OFF_CODES = kStages * B;
-    static constexpr int OFF_META = OFF_CODES + kCodes * CODES;
+    static constexpr int OFF_CODES = kX * B;
+    static constexpr int CSLOT = CODES * kCPS;         // one codes TMA: kCPS steps
+    static constexpr int OFF_META = OFF_CODES + kCodeSlots * CSLOT;
     static constexpr int OFF_BARS = OFF_META + kCodes * META;
-    static constexpr int BYTES = OFF_BARS + 256 + 1024 /* align */;
+    static constexpr int BYTES = OFF_BARS + 512 + 1024 /* barriers + TMEM slot; align */;
 };
+static_assert((2 * kCodes + 2 * kX + 2 * kStages + 1) * 8 + 4 <= 512, "barrier area");
 template <int BN>
 struct Tmem {
     static constexpr int ACC = BN;                     // accumulator columns (fp32)
@@ -148,8 +159,9 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
     const uint32_t sbase = smem_u32(smem);
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem + S::OFF_BARS);
     uint64_t *c_full = bars, *c_empty = bars + kCodes;                    // codes ring
-    uint64_t *x_full = bars + 2 * kCodes, *a_full = x_full + kStages;     // operand stages
-    uint64_t *ab_empty = a_full + kStages, *done = ab_empty + kStages;
+    uint64_t *x_full = bars + 2 * kCodes, *x_empty = x_full + kX;        // B stages (smem)
+    uint64_t *a_full = x_empty + kX, *ab_empty = a_full + kStages;        // A stages (TMEM)
+    uint64_t *done = ab_empty + kStages;
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(done + 1);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -163,8 +175,11 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
             mbar_init(&c_full[s], 1);
             mbar_init(&c_empty[s], kProd);
         }
-        for (int s = 0; s < kStages; ++s) {
+        for (int s = 0; s < kX; ++s) {
             mbar_init(&x_full[s], 1);
+            mbar_init(&x_empty[s], 1);
+        }
+        for (int s = 0; s < kStages; ++s) {
             mbar_init(&a_full[s], kProd);
             mbar_init(&ab_empty[s], 1);
         }
@@ -184,21 +199,21 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
     if (warp == kWTC) {
         // ------------------------------------------------------ TMA: q4 codes
         if (lane == 0) {
-            for (int j = 0; j < nsteps; ++j) {
-                const int cs = j % kCodes;
-                if (j >= kCodes) mbar_wait(&c_empty[cs], ((j / kCodes) - 1) & 1);
-                mbar_arrive_expect_tx(&c_full[cs], S::CODES);
-                tma_2d(sbase + S::OFF_CODES + cs * S::CODES, &tm_codes, (kb0 + j) * 32, n0, &c_full[cs]);
+            for (int q = 0; q * kCPS < nsteps; ++q) {
+                const int cs = q % kCodeSlots;
+                if (q >= kCodeSlots) mbar_wait(&c_empty[cs], ((q / kCodeSlots) - 1) & 1);
+                mbar_arrive_expect_tx(&c_full[cs], S::CSLOT);
+                tma_2d(sbase + S::OFF_CODES + cs * S::CSLOT, &tm_codes, (kb0 + q * kCPS) * 32, n0, &c_full[cs]);
             }
         }
     } else if (warp == kWTX) {
         // ------------------------------------------------------ TMA: activations
         if (lane == 0) {
             for (int j = 0; j < nsteps; ++j) {
-                const int st = j % kStages;
-                if (j >= kStages) mbar_wait(&ab_empty[st], ((j / kStages) - 1) & 1);
-                mbar_arrive_expect_tx(&x_full[st], S::B);
-                tma_2d(sbase + st * S::B, &tm_x, (kb0 + j) * kK, 0, &x_full[st]);
+                const int xs = j % kX;
+                if (j >= kX) mbar_wait(&x_empty[xs], ((j / kX) - 1) & 1);
+                mbar_arrive_expect_tx(&x_full[xs], S::B);
+                tma_2d(sbase + xs * S::B, &tm_x, (kb0 + j) * kK, 0, &x_full[xs]);
             }
         }
     } else if (warp < kWMMA) {
@@ -213,12 +228,14 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
         };
         for (int j = 0; j < kCodes - 1; ++j) meta_issue(j);
         const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16) + TM::A0 + h * (WPT / 2);
-        for (int j = 0; j < nsteps; ++j) {
+        // software pipeline: the dequant of step j overlaps the TMEM store of step j-1
+        // (tcgen05.wait::st of j-1 only after step j's arithmetic); two register buffers
+        auto produce = [&](int j, uint4 (&v)[WPT / 8]) {
             meta_issue(j + kCodes - 1);
-            const int cs = j % kCodes, st = j % kStages;
-            mbar_wait(&c_full[cs], (j / kCodes) & 1);
+            const int q = j / kCPS, cs = q % kCodeSlots, sub = j - q * kCPS;
+            if (sub == 0) mbar_wait(&c_full[cs], (q / kCodeSlots) & 1);
             uint32_t cw[WPT / 8], mw;
-            const uint32_t caddr = sbase + S::OFF_CODES + cs * S::CODES + r * 32 + h * (WPT / 2);
+            const uint32_t caddr = sbase + S::OFF_CODES + cs * S::CSLOT + r * (32 * kCPS) + sub * 32 + h * (WPT / 2);
             if constexpr (WPT == 64) {
                 asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
                              : "=r"(cw[0]), "=r"(cw[1]), "=r"(cw[2]), "=r"(cw[3]) : "r"(caddr));
@@ -229,13 +246,12 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                              : "=r"(cw[0]), "=r"(cw[1]), "=r"(cw[2]), "=r"(cw[3]) : "r"(caddr));
             else
                 asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n" : "=r"(cw[0]), "=r"(cw[1]) : "r"(caddr));
-            mbar_arrive(&c_empty[cs]);
+            if (sub == kCPS - 1 || j == nsteps - 1) mbar_arrive(&c_empty[cs]);
             cp_wait<kCodes - 1>();
-            asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(meta_u32 + cs * S::META));
+            asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(meta_u32 + (j % kCodes) * S::META));
             const __half2 mn2 = __half2half2(__ushort_as_half((unsigned short)(mw & 0xFFFFu)));
             const __half2 sc2 = __half2half2(__ushort_as_half((unsigned short)(mw >> 16)));
             const __half2 sc16 = __hmul2(sc2, __half2half2(__ushort_as_half(0x2C00)));   // * 1/16
-            uint4 v[WPT / 8];
 #pragma unroll
             for (int i = 0; i < WPT / 8; ++i) {
 #if LMO_W4_NODEQ   // (experiment: pipeline / MMA bound without the dequant arithmetic)
@@ -244,6 +260,9 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                 v[i] = deq8(cw[i], sc2, sc16, mn2);
 #endif
             }
+        };
+        auto store = [&](int j, const uint4 (&v)[WPT / 8]) {
+            const int st = j % kStages;
             if (j >= kStages) mbar_wait(&ab_empty[st], ((j / kStages) - 1) & 1);
             if constexpr (WPT == 64)
                 asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
@@ -271,21 +290,39 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                              "r"(v[0].x), "r"(v[0].y), "r"(v[0].z), "r"(v[0].w), "r"(v[WPT / 8 - 1].x),
                              "r"(v[WPT / 8 - 1].y), "r"(v[WPT / 8 - 1].z), "r"(v[WPT / 8 - 1].w)
                              : "memory");
+        };
+        auto publish = [&](int j) {
             asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
             asm volatile("tcgen05.fence::before_thread_sync;\n");
-            mbar_arrive(&a_full[st]);
+            mbar_arrive(&a_full[j % kStages]);
+        };
+        uint4 va[WPT / 8], vb[WPT / 8];
+        if (nsteps > 0) {
+            produce(0, va);
+            store(0, va);
         }
+        for (int j = 1; j < nsteps; j += 2) {
+            produce(j, vb);
+            publish(j - 1);
+            store(j, vb);
+            if (j + 1 < nsteps) {
+                produce(j + 1, va);
+                publish(j);
+                store(j + 1, va);
+            }
+        }
+        if (nsteps > 0) publish(nsteps - 1);
         cp_wait<0>();
     } else {
         // ------------------------------------------------------ MMA issuer (warp 8)
         constexpr uint32_t idesc = umma_idesc<BN>();
         for (int j = 0; j < nsteps; ++j) {
-            const int st = j % kStages;
-            mbar_wait(&x_full[st], (j / kStages) & 1);
+            const int st = j % kStages, xs = j % kX;
+            mbar_wait(&x_full[xs], (j / kX) & 1);
             mbar_wait(&a_full[st], (j / kStages) & 1);
             asm volatile("tcgen05.fence::after_thread_sync;\n");
             if (lane == 0) {
-                const uint32_t b0 = sbase + st * S::B;
+                const uint32_t b0 = sbase + xs * S::B;
 #pragma unroll
                 for (int k = 0; k < kK / 16; ++k) {
                     const uint32_t ta = tmem + TM::A0 + st * 32 + k * 8;
@@ -298,6 +335,9 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                 }
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
                                  smem_u32(&ab_empty[st]))
+                             : "memory");
+                asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
+                                 smem_u32(&x_empty[xs]))
                              : "memory");
             }
             __syncwarp();
@@ -384,10 +424,10 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const void *x, 
     if (!enc) return cudaErrorNotSupported;
     const int BN = batch <= 64 ? 64 : 128;
     CUtensorMap tc, tx;
-    {   // codes [N][K/2] u8, box 32 B x 128 rows
+    {   // codes [N][K/2] u8, box 32*kCPS B x 128 rows (out-of-range columns zero-filled)
         const cuuint64_t dims[2] = {(cuuint64_t)K / 2, (cuuint64_t)N};
         const cuuint64_t strides[1] = {(cuuint64_t)K / 2};
-        const cuuint32_t box[2] = {32, (cuuint32_t)w4::kM}, es[2] = {1, 1};
+        const cuuint32_t box[2] = {32 * w4::kCPS, (cuuint32_t)w4::kM}, es[2] = {1, 1};
         if (enc(&tc, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t *>(codes), dims, strides, box, es,
                 CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)

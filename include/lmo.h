@@ -264,6 +264,21 @@ lmo_status lmo_w4a16_linear(const uint8_t *codes, const lmo_qmeta *meta, int64_t
                             const void *x_f16, int32_t batch, float *y_f32, int32_t k_split,
                             void *stream);
 
+/* NEXT-3, streaming layout.  The paper quantizes the weights once at load
+ * time; lmo_w4a16_pack rearranges them once into the layout the GEMM
+ * streams: for each 128-row tile t and group g, one contiguous 4608-byte block
+ * at offset (t * K/64 + g) * 4608 holding the tile's 128 rows x 32 code bytes
+ * followed by their 128 lmo_qmeta.  A tile-step is then one 1-D bulk copy of
+ * whole DRAM pages instead of 128 scattered 32-byte row pieces.
+ * lmo_w4a16_packed_bytes gives the size (0 for an invalid shape);
+ * lmo_w4a16_linear_packed computes exactly what lmo_w4a16_linear computes on
+ * the unpacked codes/meta (same arithmetic, same shapes and errors). */
+size_t lmo_w4a16_packed_bytes(int64_t N, int64_t K);
+lmo_status lmo_w4a16_pack(const uint8_t *codes, const lmo_qmeta *meta, int64_t N, int64_t K,
+                          uint8_t *packed, void *stream);
+lmo_status lmo_w4a16_linear_packed(const uint8_t *packed, int64_t N, int64_t K, const void *x_f16,
+                                   int32_t batch, float *y_f32, int32_t k_split, void *stream);
+
 /* Human-readable name of a status code (static string). */
 const char *lmo_status_string(lmo_status status);
 

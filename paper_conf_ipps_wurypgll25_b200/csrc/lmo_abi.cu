@@ -48,8 +48,9 @@ bool pdl_enabled() {
 cudaError_t launch_gen_fill(void *, int, int, int, int, uint64_t, int, int, int, int, int, int,
                             cudaStream_t);
 size_t attn_workspace_bytes(int B, int Hkv, int Hq, int D, int num_splits);
-cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const void *x, float *y, int N, int K,
-                         int batch, int ksplit, cudaStream_t st);
+cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *packed, const void *x, float *y,
+                         int N, int K, int batch, int ksplit, cudaStream_t st);
+cudaError_t launch_w4a16_pack(const uint8_t *codes, const void *meta, uint8_t *packed, int N, int K, cudaStream_t st);
 
 static bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
@@ -212,7 +213,31 @@ lmo_status lmo_w4a16_linear(const uint8_t *codes, const lmo_qmeta *meta, int64_t
     if (N % 128 != 0 || K % kGroup != 0 || N > (1ll << 30) || K > (1ll << 30)) return LMO_ERR_SHAPE;
     if (batch > 128) return LMO_ERR_UNSUPPORTED;
     if (!aligned16(codes) || !aligned16(meta) || !aligned16(x) || !aligned16(y)) return LMO_ERR_ALIGN;
-    return cuda_status(launch_w4a16(codes, meta, x, y, (int)N, (int)K, batch, k_split,
+    return cuda_status(launch_w4a16(codes, meta, nullptr, x, y, (int)N, (int)K, batch, k_split,
+                                    static_cast<cudaStream_t>(stream)));
+}
+
+size_t lmo_w4a16_packed_bytes(int64_t N, int64_t K) {
+    if (N <= 0 || K <= 0 || N % 128 != 0 || K % kGroup != 0) return 0;
+    return (size_t)(N / 128) * (size_t)(K / kGroup) * 4608u;
+}
+
+lmo_status lmo_w4a16_pack(const uint8_t *codes, const lmo_qmeta *meta, int64_t N, int64_t K, uint8_t *packed,
+                          void *stream) {
+    if (!codes || !meta || !packed) return LMO_ERR_NULL;
+    if (N <= 0 || K <= 0 || N % 128 != 0 || K % kGroup != 0 || N > (1ll << 30) || K > (1ll << 30)) return LMO_ERR_SHAPE;
+    if (!aligned16(codes) || !aligned16(meta) || !aligned16(packed)) return LMO_ERR_ALIGN;
+    return cuda_status(launch_w4a16_pack(codes, meta, packed, (int)N, (int)K, static_cast<cudaStream_t>(stream)));
+}
+
+lmo_status lmo_w4a16_linear_packed(const uint8_t *packed, int64_t N, int64_t K, const void *x, int32_t batch,
+                                   float *y, int32_t k_split, void *stream) {
+    if (!packed || !x || !y) return LMO_ERR_NULL;
+    if (N <= 0 || K <= 0 || batch <= 0 || k_split < 0) return LMO_ERR_SHAPE;
+    if (N % 128 != 0 || K % kGroup != 0 || N > (1ll << 30) || K > (1ll << 30)) return LMO_ERR_SHAPE;
+    if (batch > 128) return LMO_ERR_UNSUPPORTED;
+    if (!aligned16(packed) || !aligned16(x) || !aligned16(y)) return LMO_ERR_ALIGN;
+    return cuda_status(launch_w4a16(nullptr, nullptr, packed, x, y, (int)N, (int)K, batch, k_split,
                                     static_cast<cudaStream_t>(stream)));
 }
 

@@ -34,6 +34,8 @@
 // Split-K (grid.y) accumulates fp32 partial tiles with red.global.add.
 #include <cuda.h>
 
+#include <algorithm>
+
 #include "common.cuh"
 
 namespace lmo {
@@ -54,7 +56,7 @@ constexpr int kCodes = LMO_W4_CODES;     // q4 code staging depth (steps in flig
 #endif
 constexpr int kX = LMO_W4_XSTAGES;       // B (activation) stages in smem: prefetched further ahead than A
 #ifndef LMO_W4_CPS
-#define LMO_W4_CPS 1
+#define LMO_W4_CPS 1   // (packed path: 1, 2, 4 measured equal within 2%)
 #endif
 constexpr int kCPS = LMO_W4_CPS;         // steps per codes TMA (box 32*kCPS B x 128 rows: full lines)
 constexpr int kCodeSlots = kCodes / kCPS;
@@ -76,7 +78,8 @@ struct Smem {
     static constexpr int CODES = kM * 32;              // 4 KB per step
     static constexpr int META = kM * 4 * kParts;       // per step: one 4-B copy per thread (thread-private)
     static constexpr int OFF_CODES = kX * B;
-    static constexpr int CSLOT = CODES * kCPS;         // one codes TMA: kCPS steps
+    static constexpr int PSTEP = CODES + kM * 4;       // packed layout: one step = codes | meta (4608 B)
+    static constexpr int CSLOT = PSTEP * kCPS;         // one codes transfer: kCPS steps
     static constexpr int OFF_META = OFF_CODES + kCodeSlots * CSLOT;
     static constexpr int OFF_BARS = OFF_META + kCodes * META;
     static constexpr int BYTES = OFF_BARS + 512 + 1024 /* barriers + TMEM slot; align */;
@@ -148,10 +151,14 @@ __device__ __forceinline__ void tma_2d(uint32_t dst, const void *tmap, int c0, i
         : "memory");
 }
 
-template <int BN>
+// PACKED: W in the streaming layout of lmo_w4a16_pack -- per (128-row tile, group) one
+// contiguous 4608-B block [128 rows x 32 B codes | 128 x 4 B meta], fetched with one 1-D
+// bulk copy (full DRAM pages) instead of a 2-D TMA of 128 scattered 32-B row pieces.
+template <int BN, bool PACKED>
 __global__ void __launch_bounds__(kThreads, 1)
 w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant__ CUtensorMap tm_x,
-             const uint32_t *__restrict__ meta, float *__restrict__ y, int N, int K, int batch, int ksplit) {
+             const uint32_t *__restrict__ meta, const uint8_t *__restrict__ packed, float *__restrict__ y, int N,
+             int K, int batch, int ksplit) {
     using S = Smem<BN>;
     using TM = Tmem<BN>;
     extern __shared__ uint8_t smem_raw[];
@@ -202,8 +209,15 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
             for (int q = 0; q * kCPS < nsteps; ++q) {
                 const int cs = q % kCodeSlots;
                 if (q >= kCodeSlots) mbar_wait(&c_empty[cs], ((q / kCodeSlots) - 1) & 1);
-                mbar_arrive_expect_tx(&c_full[cs], S::CSLOT);
-                tma_2d(sbase + S::OFF_CODES + cs * S::CSLOT, &tm_codes, (kb0 + q * kCPS) * 32, n0, &c_full[cs]);
+                if constexpr (PACKED) {
+                    const int ns = min(kCPS, nsteps - q * kCPS);
+                    const uint8_t *src = packed + ((int64_t)blockIdx.x * KB + kb0 + q * kCPS) * S::PSTEP;
+                    mbar_arrive_expect_tx(&c_full[cs], ns * S::PSTEP);
+                    bulk_g2s(smem + S::OFF_CODES + cs * S::CSLOT, src, ns * S::PSTEP, &c_full[cs], policy_evict_first());
+                } else {
+                    mbar_arrive_expect_tx(&c_full[cs], S::CODES * kCPS);
+                    tma_2d(sbase + S::OFF_CODES + cs * S::CSLOT, &tm_codes, (kb0 + q * kCPS) * 32, n0, &c_full[cs]);
+                }
             }
         }
     } else if (warp == kWTX) {
@@ -223,6 +237,7 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
         const uint32_t *mrow = meta + (int64_t)(n0 + r) * (K / kK);
         const uint32_t meta_u32 = sbase + S::OFF_META + (h * kM + r) * 4;
         auto meta_issue = [&](int j) {   // thread-private cp.async ring of the group meta words
+            if (PACKED) return;
             if (j < nsteps) cp_async4(meta_u32 + (j % kCodes) * S::META, mrow + kb0 + j);
             cp_commit();
         };
@@ -235,7 +250,8 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
             const int q = j / kCPS, cs = q % kCodeSlots, sub = j - q * kCPS;
             if (sub == 0) mbar_wait(&c_full[cs], (q / kCodeSlots) & 1);
             uint32_t cw[WPT / 8], mw;
-            const uint32_t caddr = sbase + S::OFF_CODES + cs * S::CSLOT + r * (32 * kCPS) + sub * 32 + h * (WPT / 2);
+            const uint32_t caddr = PACKED ? sbase + S::OFF_CODES + cs * S::CSLOT + sub * S::PSTEP + r * 32 + h * (WPT / 2)
+                                          : sbase + S::OFF_CODES + cs * S::CSLOT + r * (32 * kCPS) + sub * 32 + h * (WPT / 2);
             if constexpr (WPT == 64) {
                 asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
                              : "=r"(cw[0]), "=r"(cw[1]), "=r"(cw[2]), "=r"(cw[3]) : "r"(caddr));
@@ -246,9 +262,14 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                              : "=r"(cw[0]), "=r"(cw[1]), "=r"(cw[2]), "=r"(cw[3]) : "r"(caddr));
             else
                 asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n" : "=r"(cw[0]), "=r"(cw[1]) : "r"(caddr));
+            if constexpr (PACKED) {
+                asm volatile("ld.shared.u32 %0, [%1];\n"
+                             : "=r"(mw) : "r"(sbase + S::OFF_CODES + cs * S::CSLOT + sub * S::PSTEP + S::CODES + r * 4));
+            } else {
+                cp_wait<kCodes - 1>();
+                asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(meta_u32 + (j % kCodes) * S::META));
+            }
             if (sub == kCPS - 1 || j == nsteps - 1) mbar_arrive(&c_empty[cs]);
-            cp_wait<kCodes - 1>();
-            asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(meta_u32 + (j % kCodes) * S::META));
             const __half2 mn2 = __half2half2(__ushort_as_half((unsigned short)(mw & 0xFFFFu)));
             const __half2 sc2 = __half2half2(__ushort_as_half((unsigned short)(mw >> 16)));
             const __half2 sc16 = __hmul2(sc2, __half2half2(__ushort_as_half(0x2C00)));   // * 1/16
@@ -416,23 +437,47 @@ static EncodeTiledFn encode_tiled() {
     return fn;
 }
 
-cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const void *x, float *y, int N, int K,
-                         int batch, int ksplit, cudaStream_t st) {
+// Pack W (codes [N][K/2], meta [N][K/64]) into the streaming layout: block (tile, g) of
+// 4608 B = [128 rows x 32 B codes | 128 x 4 B meta] at ((tile * K/64) + g) * 4608.
+__global__ void w4a16_pack_kernel(const uint8_t *__restrict__ codes, const uint32_t *__restrict__ meta,
+                                  uint8_t *__restrict__ packed, int N, int K) {
+    const int KB = K / w4::kK;
+    const int64_t nchunks = (int64_t)(N / w4::kM) * KB * (w4::kM * 2 + w4::kM / 4);   // 16-B chunks
+    for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c < nchunks; c += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t blk = c / (w4::kM * 2 + w4::kM / 4);
+        const int w = (int)(c - blk * (w4::kM * 2 + w4::kM / 4));
+        const int tile = (int)(blk / KB), g = (int)(blk - (int64_t)tile * KB);
+        uint4 v;
+        if (w < w4::kM * 2) {              // codes: row w/2, half w%2
+            const int r = w >> 1, hh = w & 1;
+            v = *reinterpret_cast<const uint4 *>(codes + (int64_t)(tile * w4::kM + r) * (K / 2) + g * 32 + hh * 16);
+        } else {                           // meta: rows 4(w-256) .. +3
+            const int r0 = (w - w4::kM * 2) * 4;
+            const uint32_t *mp = meta + (int64_t)(tile * w4::kM + r0) * KB + g;
+            v = make_uint4(mp[0], mp[KB], mp[2 * KB], mp[3 * KB]);
+        }
+        *reinterpret_cast<uint4 *>(packed + blk * 4608 + (int64_t)w * 16) = v;
+    }
+}
+
+cudaError_t launch_w4a16_pack(const uint8_t *codes, const void *meta, uint8_t *packed, int N, int K, cudaStream_t st) {
+    const int64_t nchunks = (int64_t)(N / w4::kM) * (K / w4::kK) * (w4::kM * 2 + w4::kM / 4);
+    const int grid = (int)std::min<int64_t>((nchunks + 255) / 256, (int64_t)device_sm_count() * 16);
+    w4a16_pack_kernel<<<grid, 256, 0, st>>>(codes, static_cast<const uint32_t *>(meta), packed, N, K);
+    const cudaError_t e = cudaGetLastError();
+    if (e == cudaSuccess) note_launch();
+    return e;
+}
+
+// codes/meta (row-major, 2-D TMA path) or packed (streaming layout, 1-D bulk path)
+cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *packed, const void *x, float *y,
+                         int N, int K, int batch, int ksplit, cudaStream_t st) {
     if (ksplit <= 0) ksplit = w4a16_auto_split(N, K);
     if (ksplit > K / w4::kK) ksplit = K / w4::kK;
     EncodeTiledFn enc = encode_tiled();
     if (!enc) return cudaErrorNotSupported;
     const int BN = batch <= 64 ? 64 : 128;
     CUtensorMap tc, tx;
-    {   // codes [N][K/2] u8, box 32*kCPS B x 128 rows (out-of-range columns zero-filled)
-        const cuuint64_t dims[2] = {(cuuint64_t)K / 2, (cuuint64_t)N};
-        const cuuint64_t strides[1] = {(cuuint64_t)K / 2};
-        const cuuint32_t box[2] = {32 * w4::kCPS, (cuuint32_t)w4::kM}, es[2] = {1, 1};
-        if (enc(&tc, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t *>(codes), dims, strides, box, es,
-                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
-            return cudaErrorInvalidValue;
-    }
     {   // x [batch][K] fp16, box 64 x BN rows, SWIZZLE_128B (rows >= batch are zero-filled)
         const cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)batch};
         const cuuint64_t strides[1] = {(cuuint64_t)K * 2};
@@ -442,20 +487,33 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const void *x, 
                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
             return cudaErrorInvalidValue;
     }
+    if (packed) {
+        tc = tx;                                                   // (unused by the packed path)
+    } else {   // codes [N][K/2] u8, box 32*kCPS B x 128 rows (out-of-range columns zero-filled)
+        const cuuint64_t dims[2] = {(cuuint64_t)K / 2, (cuuint64_t)N};
+        const cuuint64_t strides[1] = {(cuuint64_t)K / 2};
+        const cuuint32_t box[2] = {32 * w4::kCPS, (cuuint32_t)w4::kM}, es[2] = {1, 1};
+        if (enc(&tc, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t *>(codes), dims, strides, box, es,
+                CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+            return cudaErrorInvalidValue;
+    }
     if (ksplit > 1) {
         const cudaError_t e = cudaMemsetAsync(y, 0, (size_t)batch * N * sizeof(float), st);
         if (e != cudaSuccess) return e;
     }
     dim3 grid(N / w4::kM, ksplit);
     const uint32_t *m = static_cast<const uint32_t *>(meta);
+    auto go = [&](auto kern, int sm) {
+        cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+        kern<<<grid, w4::kThreads, sm, st>>>(tc, tx, m, packed, y, N, K, batch, ksplit);
+    };
     if (BN == 64) {
-        const int sm = w4::Smem<64>::BYTES;
-        cudaFuncSetAttribute(w4::w4a16_kernel<64>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
-        w4::w4a16_kernel<64><<<grid, w4::kThreads, sm, st>>>(tc, tx, m, y, N, K, batch, ksplit);
+        if (packed) go(w4::w4a16_kernel<64, true>, w4::Smem<64>::BYTES);
+        else go(w4::w4a16_kernel<64, false>, w4::Smem<64>::BYTES);
     } else {
-        const int sm = w4::Smem<128>::BYTES;
-        cudaFuncSetAttribute(w4::w4a16_kernel<128>, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
-        w4::w4a16_kernel<128><<<grid, w4::kThreads, sm, st>>>(tc, tx, m, y, N, K, batch, ksplit);
+        if (packed) go(w4::w4a16_kernel<128, true>, w4::Smem<128>::BYTES);
+        else go(w4::w4a16_kernel<128, false>, w4::Smem<128>::BYTES);
     }
     const cudaError_t e = cudaGetLastError();
     if (e == cudaSuccess) note_launch();

@@ -50,6 +50,8 @@ def _load():
                                     i32, P, ctypes.c_int, P, ctypes.c_size_t, P],
         "lmo_gen_fill_f16": [P, i32, i32, i32, i32, u64, i32, i32, i32, i32, i32, i32, P],
         "lmo_w4a16_linear": [P, P, i64, i64, P, i32, P, i32, P],
+        "lmo_w4a16_pack": [P, P, i64, i64, P, P],
+        "lmo_w4a16_linear_packed": [P, i64, i64, P, i32, P, i32, P],
         "lmo_decode_step_q4": [ctypes.POINTER(lmo_kv_cache), P, P, P, i32, i32, P, ctypes.c_float,
                                i32, P, ctypes.c_int, P, ctypes.c_size_t, ctypes.c_uint32, P],
     }
@@ -70,6 +72,8 @@ def _load():
     L.lmo_decode_attention_workspace_bytes.restype = ctypes.c_size_t
     L.lmo_status_string.argtypes = [ctypes.c_int]
     L.lmo_status_string.restype = ctypes.c_char_p
+    L.lmo_w4a16_packed_bytes.argtypes = [i64, i64]
+    L.lmo_w4a16_packed_bytes.restype = ctypes.c_size_t
     L.lmo_kv_row_bytes.argtypes = [i32]
     L.lmo_kv_row_bytes.restype = ctypes.c_size_t
     L.lmo_launch_count.argtypes = []
@@ -87,7 +91,8 @@ EXPORTS = ["lmo_quantize_groupwise", "lmo_dequantize_groupwise", "lmo_kv_append_
            "lmo_status_string",
            "lmo_gen_fill_f16", "lmo_launch_count", "lmo_version",
            "lmo_offload_ring_bytes", "lmo_offload_create", "lmo_offload_decode_step",
-           "lmo_offload_destroy", "lmo_w4a16_linear"]
+           "lmo_offload_destroy", "lmo_w4a16_linear", "lmo_w4a16_packed_bytes", "lmo_w4a16_pack",
+           "lmo_w4a16_linear_packed"]
 
 
 def _check(status: int, fn: str) -> None:
@@ -157,6 +162,29 @@ def lmo_w4a16_linear(codes: torch.Tensor, meta: torch.Tensor, N: int, K: int, x:
     _need_cuda(codes, meta, x, y)
     _check(_lib.lmo_w4a16_linear(_ptr(codes), _ptr(meta), N, K, _ptr(x), batch, _ptr(y), k_split,
                                  _stream(stream)), "lmo_w4a16_linear")
+    return y
+
+
+def lmo_w4a16_pack(codes: torch.Tensor, meta: torch.Tensor, N: int, K: int, stream=None) -> torch.Tensor:
+    """Once-per-weight repack into the GEMM's streaming layout (include/lmo.h)."""
+    nbytes = _lib.lmo_w4a16_packed_bytes(N, K)
+    if nbytes == 0:
+        raise LmoError(LMO_ERR_SHAPE, "lmo_w4a16_packed_bytes")
+    packed = torch.empty(nbytes, dtype=torch.uint8, device=codes.device)
+    _need_cuda(codes, meta, packed)
+    _check(_lib.lmo_w4a16_pack(_ptr(codes), _ptr(meta), N, K, _ptr(packed), _stream(stream)), "lmo_w4a16_pack")
+    return packed
+
+
+def lmo_w4a16_linear_packed(packed: torch.Tensor, N: int, K: int, x: torch.Tensor,
+                            y: torch.Tensor | None = None, k_split: int = 0, stream=None) -> torch.Tensor:
+    """lmo_w4a16_linear on weights in the packed streaming layout."""
+    batch = x.numel() // K
+    if y is None:
+        y = torch.empty((batch, N), dtype=torch.float32, device=x.device)
+    _need_cuda(packed, x, y)
+    _check(_lib.lmo_w4a16_linear_packed(_ptr(packed), N, K, _ptr(x), batch, _ptr(y), k_split, _stream(stream)),
+           "lmo_w4a16_linear_packed")
     return y
 
 

@@ -6,6 +6,7 @@ import torch
 from paper_conf_ipps_wurypgll25_b200 import lmo
 
 split = int(sys.argv[1]) if len(sys.argv) > 1 else 0
+PACKED = os.environ.get("PACKED", "1") == "1"
 h1, B = 7168, 64
 shapes = {"qkv": (3 * h1, h1), "o": (h1, h1), "ffn1": (4 * h1, h1), "ffn2": (h1, 4 * h1)}
 tot_t = tot_b = 0
@@ -13,17 +14,18 @@ for name, (N, K) in shapes.items():
     W = (torch.randn(N, K, device="cuda") * 0.02).half()
     codes, meta = lmo.lmo_quantize_groupwise(W, N, K, 1)
     codes, meta = codes.view(N, K // 2), meta.view(N, K // 64)
+    packed = lmo.lmo_w4a16_pack(codes, meta, N, K) if PACKED else None
     x = torch.randn(B, K, device="cuda").half()
     y = torch.empty(B, N, device="cuda")
     nrep = 20
     # several weight copies would exceed nothing here: one layer's weights >> L2 per GEMM for qkv/ffn
     for _ in range(3):
-        lmo.lmo_w4a16_linear(codes, meta, N, K, x, y=y, k_split=split)
+        (lmo.lmo_w4a16_linear_packed(packed, N, K, x, y=y, k_split=split) if PACKED else lmo.lmo_w4a16_linear(codes, meta, N, K, x, y=y, k_split=split))
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record()
     for _ in range(nrep):
-        lmo.lmo_w4a16_linear(codes, meta, N, K, x, y=y, k_split=split)
+        (lmo.lmo_w4a16_linear_packed(packed, N, K, x, y=y, k_split=split) if PACKED else lmo.lmo_w4a16_linear(codes, meta, N, K, x, y=y, k_split=split))
     e1.record(); torch.cuda.synchronize()
     us = e0.elapsed_time(e1) * 1e3 / nrep
     by = N * K * 0.5 + N * (K // 64) * 4 + B * K * 2 + B * N * 4

@@ -128,3 +128,30 @@ def test_w4a16_argument_errors(lmo):
     xb = torch.zeros((129, 64), dtype=torch.float16, device="cuda")
     with pytest.raises(lmo.LmoError):
         lmo.lmo_w4a16_linear(c, m, 128, 64, xb)                    # batch > 128
+
+
+@pytest.mark.parametrize("N,K,batch,k_split", [(128, 64, 3, 1), (256, 320, 5, 2), (384, 1024, 64, 0),
+                                                (256, 512, 100, 3)])
+def test_w4a16_packed_layout(lmo, N, K, batch, k_split):
+    """lmo_w4a16_pack + lmo_w4a16_linear_packed: the packed blocks hold exactly the
+    tile's codes then its meta words, and the packed GEMM is bit-identical to the
+    row-major one (same arithmetic, same split) and within the oracle bound."""
+    rng = np.random.default_rng(2000 + N + K + batch)
+    codes, meta = make_weights(rng, N, K)
+    c, m = torch.from_numpy(codes).cuda(), torch.from_numpy(meta.view(np.int32)).cuda()
+    packed = lmo.lmo_w4a16_pack(c, m, N, K).cpu().numpy()
+    KB = K // 64
+    blk = packed.reshape(N // 128, KB, 4608)
+    for t in range(N // 128):
+        for g in (0, KB - 1):
+            assert np.array_equal(blk[t, g, :4096].reshape(128, 32), codes[t * 128:(t + 1) * 128, g * 32:(g + 1) * 32])
+            assert np.array_equal(blk[t, g, 4096:].view(np.uint16).reshape(128, 2), meta[t * 128:(t + 1) * 128, g])
+    x = torch.from_numpy(rng.standard_normal((batch, K)).astype(np.float16)).cuda()
+    y1 = lmo.lmo_w4a16_linear(c, m, N, K, x, k_split=1).cpu()
+    yp = lmo.lmo_w4a16_linear_packed(torch.from_numpy(packed).cuda(), N, K, x, k_split=1).cpu()
+    assert torch.equal(y1, yp)
+    ys = lmo.lmo_w4a16_linear_packed(torch.from_numpy(packed).cuda(), N, K, x, k_split=k_split).cpu().numpy()
+    ref = oracle.w4a16_linear(codes, meta, N, K, x.cpu().numpy())
+    wdq = oracle.dequantize_groupwise(codes, meta, N, K, 1).reshape(N, K).astype(np.float64)
+    bound = np.abs(x.cpu().numpy().astype(np.float64)) @ np.abs(wdq).T * 2.0 ** -10 + 1e-6
+    assert np.all(np.abs(ys - ref) <= bound)

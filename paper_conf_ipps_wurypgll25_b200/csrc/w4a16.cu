@@ -60,6 +60,9 @@ constexpr int kX = LMO_W4_XSTAGES;       // B (activation) stages in smem: prefe
 #endif
 constexpr int kCPS = LMO_W4_CPS;         // steps per codes TMA (box 32*kCPS B x 128 rows: full lines)
 constexpr int kCodeSlots = kCodes / kCPS;
+#ifndef LMO_W4_WARP_ARRIVE
+#define LMO_W4_WARP_ARRIVE 0   // 1: one mbarrier arrival per producer warp (measured equal)
+#endif
 #ifndef LMO_W4_NODEQ
 #define LMO_W4_NODEQ 0
 #endif
@@ -180,14 +183,14 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
     if (tid == 0) {
         for (int s = 0; s < kCodes; ++s) {
             mbar_init(&c_full[s], 1);
-            mbar_init(&c_empty[s], kProd);
+            mbar_init(&c_empty[s], LMO_W4_WARP_ARRIVE ? kProd / 32 : kProd);
         }
         for (int s = 0; s < kX; ++s) {
             mbar_init(&x_full[s], 1);
             mbar_init(&x_empty[s], 1);
         }
         for (int s = 0; s < kStages; ++s) {
-            mbar_init(&a_full[s], kProd);
+            mbar_init(&a_full[s], LMO_W4_WARP_ARRIVE ? kProd / 32 : kProd);
             mbar_init(&ab_empty[s], 1);
         }
         mbar_init(done, 1);
@@ -269,7 +272,8 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                 cp_wait<kCodes - 1>();
                 asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(meta_u32 + (j % kCodes) * S::META));
             }
-            if (sub == kCPS - 1 || j == nsteps - 1) mbar_arrive(&c_empty[cs]);
+            const bool last_sub = sub == kCPS - 1 || j == nsteps - 1;
+            if (!LMO_W4_WARP_ARRIVE && last_sub) mbar_arrive(&c_empty[cs]);
             const __half2 mn2 = __half2half2(__ushort_as_half((unsigned short)(mw & 0xFFFFu)));
             const __half2 sc2 = __half2half2(__ushort_as_half((unsigned short)(mw >> 16)));
             const __half2 sc16 = __hmul2(sc2, __half2half2(__ushort_as_half(0x2C00)));   // * 1/16
@@ -280,6 +284,10 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
 #else
                 v[i] = deq8(cw[i], sc2, sc16, mn2);
 #endif
+            }
+            if (LMO_W4_WARP_ARRIVE && last_sub) {   // codes consumed (results in registers): one arrive per warp
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&c_empty[cs]);
             }
         };
         auto store = [&](int j, const uint4 (&v)[WPT / 8]) {
@@ -315,7 +323,12 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
         auto publish = [&](int j) {
             asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
             asm volatile("tcgen05.fence::before_thread_sync;\n");
-            mbar_arrive(&a_full[j % kStages]);
+            if (LMO_W4_WARP_ARRIVE) {
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&a_full[j % kStages]);
+            } else {
+                mbar_arrive(&a_full[j % kStages]);
+            }
         };
         uint4 va[WPT / 8], vb[WPT / 8];
         if (nsteps > 0) {

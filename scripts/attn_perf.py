@@ -13,7 +13,7 @@ for key in keys:
     w = CONFIGS[key]
     nl = max(2, min(16, int(2.0e9 // (w.batch * w.kv_heads * w.capacity * 144))))
     caches = []
-    L = w.max_len
+    L = int(os.environ.get("LEN", "0")) or w.max_len   # LEN: the bench's mid length s + t_mid
     for l in range(nl):
         c = lmo.KVCache.empty(w.batch, w.kv_heads, w.capacity, w.head_dim)
         c.kv.random_(0, 256)

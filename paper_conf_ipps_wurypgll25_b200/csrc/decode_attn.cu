@@ -1328,10 +1328,12 @@ __global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1
             }
             ++team_k;
         } else if (full) {
+            // (an empty sequence -- per-sequence length 0 -- keeps the zero row written at entry)
 #pragma unroll
             for (int e = 0; e < 2; ++e) {
                 const int h = 2 * t + e;
                 const float il = 1.f / lt[e];
+                if (sd.L <= 0) break;
 #pragma unroll
                 for (int grp = 0; grp < NG; ++grp) {
 #pragma unroll

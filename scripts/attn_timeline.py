@@ -94,3 +94,14 @@ for k in sorted(set(segs.tolist())):
 le = (b[:, 13] - b[:, 4].min()) / 1e3
 z2 = (b[:, 7] - b[:, 4].min()) / 1e3
 print(f"launch 2 (rel. to first entry): loop end {le.min():.2f}/{le.median():.2f}/{le.max():.2f}  kernel exit {z2.min():.2f}/{z2.median():.2f}/{z2.max():.2f} us")
+# segments (pairs) per SMSP: is the extra work concentrated on some SMSP indices?
+seg_sp = collections.Counter()
+for a, c, k in zip(sm.tolist(), sp.tolist(), segs.tolist()):
+    seg_sp[(a, c)] += k
+print("segments per SMSP:", sorted(collections.Counter(seg_sp.values()).items()))
+by_idx = collections.defaultdict(list)
+for (a, c), k in seg_sp.items():
+    by_idx[c].append(k)
+print("mean segments per SMSP index:", {c: round(sum(v) / len(v), 2) for c, v in sorted(by_idx.items())})
+# CTA -> SM placement: which CTA ids share an SM (first 8 SMs)
+cta = b[:, 3].long() & 0  # (CTA id is not recorded; warp id within SM is)

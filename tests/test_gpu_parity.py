@@ -257,6 +257,25 @@ def test_attention_per_sequence_lengths_and_reuse(lmo):
     assert int(ws[: 4 * B * Hkv].view(torch.int32).abs().sum()) == 0
 
 
+@pytest.mark.parametrize("team", [1, 2, 4])
+def test_attention_empty_sequence_every_team_size(lmo, team):
+    """A per-sequence length of 0 leaves a zero output row for every team size
+    (team 1 is the default schedule of the BASELINE configs)."""
+    B, Hkv, G, d, cap = 5, 4, 1, 128, 96
+    cache, host = build_layer(lmo, B, Hkv, cap, d, cap, 91)
+    lens = np.array([40, 0, 96, 1, 0], np.int32)
+    q = torch.empty((B, Hkv * G, 1, d), dtype=torch.float16, device="cuda")
+    lmo.lmo_gen_fill_f16(q, 91, I.STREAM_Q, 0, 0, 0, 0, group=G)
+    q = q.view(B, Hkv * G, d)
+    ws = lmo.attention_workspace(B, Hkv, Hkv * G, d, team)
+    out = lmo.lmo_decode_attention_q4(cache, q, 0, seq_lens=dev(lens), workspace=ws, num_splits=team)
+    o = out.cpu().numpy()
+    assert np.all(o[lens == 0] == 0)
+    keep = lens > 0
+    ref = oracle.decode_attention_q4(host, q.cpu().numpy(), np.maximum(lens, 1), nthreads=4)
+    assert normwise_err(o[keep], ref[keep]).max() <= TOL
+
+
 def test_attention_split_modes_agree(lmo):
     """stream-K (0) and fixed splits (1, 5) give the same result within rounding;
     a fixed split count is deterministic."""

@@ -375,8 +375,9 @@ def test_decode_step_fused_append(lmo, B, Hkv, G, d, L, ns, flags):
     assert normwise_err(out.cpu().numpy(), ref).max() <= TOL
 
 
-def test_decode_step_per_sequence_lengths(lmo):
-    B, Hkv, G, d, cap = 5, 3, 2, 128, 208
+@pytest.mark.parametrize("team,G", [(0, 2), (1, 2), (1, 1), (2, 1)])
+def test_decode_step_per_sequence_lengths(lmo, team, G):
+    B, Hkv, d, cap = 5, 3, 128, 208
     lens = np.array([200, 1, 0, 65, 129], np.int32)
     kf = torch.empty((B, Hkv, cap, d), dtype=torch.float16, device="cuda")
     vf = torch.empty_like(kf)
@@ -391,7 +392,7 @@ def test_decode_step_per_sequence_lengths(lmo):
     q = torch.empty((B, Hkv * G, 1, d), dtype=torch.float16, device="cuda")
     lmo.lmo_gen_fill_f16(q, 9, I.STREAM_Q, 0, 0, 0, 0, group=G)
     q = q.view(B, Hkv * G, d)
-    out = lmo.lmo_decode_step_q4(cache, kn, vn, q, 0, seq_lens=dev(lens))
+    out = lmo.lmo_decode_step_q4(cache, kn, vn, q, 0, seq_lens=dev(lens), num_splits=team)
     torch.cuda.synchronize()
     kh, vh = kf.cpu().numpy().copy(), vf.cpu().numpy().copy()
     for b in range(B):

@@ -293,6 +293,9 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
         auto store = [&](int j, const uint4 (&v)[WPT / 8]) {
             const int st = j % kStages;
             if (j >= kStages) mbar_wait(&ab_empty[st], ((j / kStages) - 1) & 1);
+            // order the TMEM store after the MMA that last read this A stage (WAR across the
+            // mbarrier): without it a store can overtake the wait under load
+            asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
             if constexpr (WPT == 64)
                 asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
                              "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};\n" ::"r"(lane_base + st * 32),

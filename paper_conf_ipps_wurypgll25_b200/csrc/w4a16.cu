@@ -70,30 +70,39 @@ constexpr int kCodeSlots = kCodes / kCPS;
 #define LMO_W4_PARTS 1
 #endif
 constexpr int kParts = LMO_W4_PARTS;     // dequant threads per weight row (each: 64/kParts weights per step)
-constexpr int kProd = 128 * kParts;      // dequant threads
-constexpr int kWMMA = kProd / 32;        // warp ids: MMA issuer, codes TMA, activation TMA
-constexpr int kWTC = kWMMA + 1, kWTX = kWMMA + 2;
-constexpr int kThreads = kProd + 96;
+// MT: 128-row tiles per CTA (1 or 2).  With MT = 2 one CTA covers 256 output features:
+// two accumulators and two A stages per step in TMEM share ONE activation stage, so the
+// per-step synchronisation and the activation traffic are amortised over twice the weights.
+template <int MT>
+struct Roles {
+    static constexpr int PROD = 128 * kParts * MT;     // dequant threads
+    static constexpr int WMMA = PROD / 32;             // warp ids: MMA issuer, codes TMA, activation TMA
+    static constexpr int WTC = WMMA + 1, WTX = WMMA + 2;
+    static constexpr int THREADS = PROD + 96;
+};
+constexpr int kProd = Roles<1>::PROD;   // (MT = 1 names kept for the single-tile code paths)
 
-template <int BN>
+template <int BN, int MT = 1>
 struct Smem {
     static constexpr int B = BN * 128;                 // BN x 64 fp16, SWIZZLE_128B
-    static constexpr int CODES = kM * 32;              // 4 KB per step
-    static constexpr int META = kM * 4 * kParts;       // per step: one 4-B copy per thread (thread-private)
+    static constexpr int CODES = kM * 32 * MT;         // 4 KB per tile per step
+    static constexpr int META = kM * 4 * kParts * MT;  // per step: one 4-B copy per thread (thread-private)
     static constexpr int OFF_CODES = kX * B;
-    static constexpr int PSTEP = CODES + kM * 4;       // packed layout: one step = codes | meta (4608 B)
+    static constexpr int PBLK = kM * 32 + kM * 4;      // packed layout: one tile-step = codes | meta (4608 B)
+    static constexpr int PSTEP = PBLK * MT;
     static constexpr int CSLOT = PSTEP * kCPS;         // one codes transfer: kCPS steps
     static constexpr int OFF_META = OFF_CODES + kCodeSlots * CSLOT;
     static constexpr int OFF_BARS = OFF_META + kCodes * META;
     static constexpr int BYTES = OFF_BARS + 512 + 1024 /* barriers + TMEM slot; align */;
 };
 static_assert((2 * kCodes + 2 * kX + 2 * kStages + 1) * 8 + 4 <= 512, "barrier area");
-template <int BN>
+template <int BN, int MT = 1>
 struct Tmem {
-    static constexpr int ACC = BN;                     // accumulator columns (fp32)
-    static constexpr int A0 = BN;                      // A stages: 32 columns each (64 fp16 per lane)
-    static constexpr int USED = BN + kStages * 32;
+    static constexpr int ACC = BN * MT;                // accumulator columns (fp32), tile mt at mt * BN
+    static constexpr int A0 = BN * MT;                 // A stages: 32 columns per tile (64 fp16 per lane)
+    static constexpr int USED = BN * MT + kStages * 32 * MT;
     static constexpr int COLS = USED <= 32 ? 32 : USED <= 64 ? 64 : USED <= 128 ? 128 : USED <= 256 ? 256 : 512;
+    static_assert(USED <= 512, "TMEM");
 };
 
 __device__ __forceinline__ void cp_async16(uint32_t dst, const void *src, uint32_t src_bytes) {
@@ -157,13 +166,15 @@ __device__ __forceinline__ void tma_2d(uint32_t dst, const void *tmap, int c0, i
 // PACKED: W in the streaming layout of lmo_w4a16_pack -- per (128-row tile, group) one
 // contiguous 4608-B block [128 rows x 32 B codes | 128 x 4 B meta], fetched with one 1-D
 // bulk copy (full DRAM pages) instead of a 2-D TMA of 128 scattered 32-B row pieces.
-template <int BN, bool PACKED>
-__global__ void __launch_bounds__(kThreads, 1)
+template <int BN, bool PACKED, int MT>
+__global__ void __launch_bounds__(Roles<MT>::THREADS, 1)
 w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant__ CUtensorMap tm_x,
              const uint32_t *__restrict__ meta, const uint8_t *__restrict__ packed, float *__restrict__ y, int N,
              int K, int batch, int ksplit) {
-    using S = Smem<BN>;
-    using TM = Tmem<BN>;
+    using S = Smem<BN, MT>;
+    using TM = Tmem<BN, MT>;
+    constexpr int kProd = Roles<MT>::PROD, kWMMA = Roles<MT>::WMMA, kWTC = Roles<MT>::WTC, kWTX = Roles<MT>::WTX;
+    static_assert(MT == 1 || (kParts == 1 && kCPS == 1), "two tiles per CTA: one dequant thread per row, kCPS 1");
     extern __shared__ uint8_t smem_raw[];
     uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     const uint32_t sbase = smem_u32(smem);
@@ -175,7 +186,7 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(done + 1);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int n0 = blockIdx.x * kM;
+    const int n0 = blockIdx.x * kM * MT;
     const int KB = K / kK;
     const int kb0 = (int)((long long)blockIdx.y * KB / ksplit), kb1 = (int)((long long)(blockIdx.y + 1) * KB / ksplit);
     const int nsteps = kb1 - kb0;
@@ -214,9 +225,13 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                 if (q >= kCodeSlots) mbar_wait(&c_empty[cs], ((q / kCodeSlots) - 1) & 1);
                 if constexpr (PACKED) {
                     const int ns = min(kCPS, nsteps - q * kCPS);
-                    const uint8_t *src = packed + ((int64_t)blockIdx.x * KB + kb0 + q * kCPS) * S::PSTEP;
                     mbar_arrive_expect_tx(&c_full[cs], ns * S::PSTEP);
-                    bulk_g2s(smem + S::OFF_CODES + cs * S::CSLOT, src, ns * S::PSTEP, &c_full[cs], policy_evict_first());
+#pragma unroll
+                    for (int mt = 0; mt < MT; ++mt) {
+                        const uint8_t *src = packed + ((int64_t)(blockIdx.x * MT + mt) * KB + kb0 + q * kCPS) * S::PBLK;
+                        bulk_g2s(smem + S::OFF_CODES + cs * S::CSLOT + mt * S::PBLK * kCPS, src, ns * S::PBLK,
+                                 &c_full[cs], policy_evict_first());
+                    }
                 } else {
                     mbar_arrive_expect_tx(&c_full[cs], S::CODES * kCPS);
                     tma_2d(sbase + S::OFF_CODES + cs * S::CSLOT, &tm_codes, (kb0 + q * kCPS) * 32, n0, &c_full[cs]);
@@ -236,16 +251,18 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
     } else if (warp < kWMMA) {
         // ------------------------------------------------------ dequant -> TMEM
         constexpr int WPT = kK / kParts;                        // weights per thread per step
-        const int r = tid & (kM - 1), h = tid >> 7;             // TMEM lane r (warp % 4 quarter), part h
-        const uint32_t *mrow = meta + (int64_t)(n0 + r) * (K / kK);
-        const uint32_t meta_u32 = sbase + S::OFF_META + (h * kM + r) * 4;
+        // thread -> (tile mt, row r = TMEM lane, part h); MT = 2 implies kParts = 1 (h = 0)
+        const int r = tid & (kM - 1), mt = MT == 1 ? 0 : tid >> 7, h = MT == 1 ? tid >> 7 : 0;
+        const int tr = mt * kM + r;                              // row within the CTA's rows
+        const uint32_t *mrow = meta + (int64_t)(n0 + tr) * (K / kK);
+        const uint32_t meta_u32 = sbase + S::OFF_META + (h * kM * MT + tr) * 4;
         auto meta_issue = [&](int j) {   // thread-private cp.async ring of the group meta words
             if (PACKED) return;
             if (j < nsteps) cp_async4(meta_u32 + (j % kCodes) * S::META, mrow + kb0 + j);
             cp_commit();
         };
         for (int j = 0; j < kCodes - 1; ++j) meta_issue(j);
-        const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16) + TM::A0 + h * (WPT / 2);
+        const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16) + TM::A0 + mt * 32 + h * (WPT / 2);
         // software pipeline: the dequant of step j overlaps the TMEM store of step j-1
         // (tcgen05.wait::st of j-1 only after step j's arithmetic); two register buffers
         auto produce = [&](int j, uint4 (&v)[WPT / 8]) {
@@ -253,8 +270,8 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
             const int q = j / kCPS, cs = q % kCodeSlots, sub = j - q * kCPS;
             if (sub == 0) mbar_wait(&c_full[cs], (q / kCodeSlots) & 1);
             uint32_t cw[WPT / 8], mw;
-            const uint32_t caddr = PACKED ? sbase + S::OFF_CODES + cs * S::CSLOT + sub * S::PSTEP + r * 32 + h * (WPT / 2)
-                                          : sbase + S::OFF_CODES + cs * S::CSLOT + r * (32 * kCPS) + sub * 32 + h * (WPT / 2);
+            const uint32_t caddr = PACKED ? sbase + S::OFF_CODES + cs * S::CSLOT + (mt * kCPS + sub) * S::PBLK + r * 32 + h * (WPT / 2)
+                                          : sbase + S::OFF_CODES + cs * S::CSLOT + tr * (32 * kCPS) + sub * 32 + h * (WPT / 2);
             if constexpr (WPT == 64) {
                 asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
                              : "=r"(cw[0]), "=r"(cw[1]), "=r"(cw[2]), "=r"(cw[3]) : "r"(caddr));
@@ -267,7 +284,7 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                 asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n" : "=r"(cw[0]), "=r"(cw[1]) : "r"(caddr));
             if constexpr (PACKED) {
                 asm volatile("ld.shared.u32 %0, [%1];\n"
-                             : "=r"(mw) : "r"(sbase + S::OFF_CODES + cs * S::CSLOT + sub * S::PSTEP + S::CODES + r * 4));
+                             : "=r"(mw) : "r"(sbase + S::OFF_CODES + cs * S::CSLOT + (mt * kCPS + sub) * S::PBLK + kM * 32 + r * 4));
             } else {
                 cp_wait<kCodes - 1>();
                 asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(meta_u32 + (j % kCodes) * S::META));
@@ -298,7 +315,7 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
             asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
             if constexpr (WPT == 64)
                 asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
-                             "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};\n" ::"r"(lane_base + st * 32),
+                             "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};\n" ::"r"(lane_base + st * 32 * MT),
                              "r"(v[0].x), "r"(v[0].y), "r"(v[0].z), "r"(v[0].w), "r"(v[1].x), "r"(v[1].y), "r"(v[1].z),
                              "r"(v[1].w), "r"(v[2 % (WPT / 8)].x), "r"(v[2 % (WPT / 8)].y), "r"(v[2 % (WPT / 8)].z),
                              "r"(v[2 % (WPT / 8)].w), "r"(v[3 % (WPT / 8)].x), "r"(v[3 % (WPT / 8)].y),
@@ -311,14 +328,14 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                              : "memory");
             else if constexpr (WPT == 32)
                 asm volatile("tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};\n" ::"r"(
-                                 lane_base + st * 32),
+                                 lane_base + st * 32 * MT),
                              "r"(v[0].x), "r"(v[0].y), "r"(v[0].z), "r"(v[0].w), "r"(v[1].x), "r"(v[1].y), "r"(v[1].z),
                              "r"(v[1].w), "r"(v[WPT / 8 - 2].x), "r"(v[WPT / 8 - 2].y), "r"(v[WPT / 8 - 2].z),
                              "r"(v[WPT / 8 - 2].w), "r"(v[WPT / 8 - 1].x), "r"(v[WPT / 8 - 1].y), "r"(v[WPT / 8 - 1].z),
                              "r"(v[WPT / 8 - 1].w)
                              : "memory");
             else
-                asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};\n" ::"r"(lane_base + st * 32),
+                asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};\n" ::"r"(lane_base + st * 32 * MT),
                              "r"(v[0].x), "r"(v[0].y), "r"(v[0].z), "r"(v[0].w), "r"(v[WPT / 8 - 1].x),
                              "r"(v[WPT / 8 - 1].y), "r"(v[WPT / 8 - 1].z), "r"(v[WPT / 8 - 1].w)
                              : "memory");
@@ -361,13 +378,15 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
             if (lane == 0) {
                 const uint32_t b0 = sbase + xs * S::B;
 #pragma unroll
+                for (int mt = 0; mt < MT; ++mt)
+#pragma unroll
                 for (int k = 0; k < kK / 16; ++k) {
-                    const uint32_t ta = tmem + TM::A0 + st * 32 + k * 8;
+                    const uint32_t ta = tmem + TM::A0 + (st * MT + mt) * 32 + k * 8;
                     const uint64_t db = umma_desc(b0 + k * 32);
                     const uint32_t acc = (j > 0 || k > 0) ? 1u : 0u;
                     asm volatile(
                         "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-                        "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem),
+                        "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem + mt * BN),
                         "r"(ta), "l"(db), "r"(idesc), "r"(acc));
                 }
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
@@ -387,8 +406,9 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
     }
 
     // ---------------------------------------------------------------- epilogue
-    if (warp < 4) {
-        const int row = warp * 32 + lane;                        // TMEM lane = output feature
+    if (warp < 4 * MT) {
+        const int emt = warp >> 2;                               // tile of this epilogue warp
+        const int row = emt * kM + (warp & 3) * 32 + lane;       // TMEM lane = output feature
         if (nsteps > 0) {
             mbar_wait(done, 0);
             asm volatile("tcgen05.fence::after_thread_sync;\n");
@@ -396,7 +416,7 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
 #pragma unroll
         for (int c0 = 0; c0 < BN; c0 += 32) {
             uint32_t v[32];
-            const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + c0;
+            const uint32_t taddr = tmem + ((uint32_t)((warp & 3) * 32) << 16) + emt * BN + c0;
             asm volatile(
                 "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
                 "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];\n"
@@ -430,12 +450,22 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
 
 }  // namespace w4
 
+#ifndef LMO_W4_MT
+#define LMO_W4_MT 1   // 2: two 128-row tiles per CTA when N % 256 == 0 (measured slower: 213 vs 190 us)
+#endif
+static int w4a16_mt(int N) { return (LMO_W4_MT == 2 && N % (2 * w4::kM) == 0) ? 2 : 1; }
+
 int w4a16_auto_split(int N, int K) {
-    const int tiles = N / w4::kM, KB = K / w4::kK;
-    const int sms = device_sm_count();
-    int s = 1;
-    while (tiles * s < sms && s * 2 <= KB / 4) s *= 2;   // fill the SMs, keep >= 4 groups per split
-    return s;
+    // the most K splits that still fit ONE wave of resident CTAs (2 per SM with one tile per
+    // CTA, 1 with two); measured on the OPT-30B layer GEMMs: more CTAs than one wave (or
+    // a half-empty last wave) costs more than the split-K atomics save
+    const int MT = w4a16_mt(N);
+    const int tiles = N / (w4::kM * MT), KB = K / w4::kK;
+    const int slots = device_sm_count() * (MT == 1 ? 2 : 1);
+    int s = slots / tiles;
+    if (s > 8) s = 8;
+    if (s > KB / 4) s = KB / 4;
+    return s < 1 ? 1 : s;
 }
 
 typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, const cuuint64_t *,
@@ -508,7 +538,7 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
     } else {   // codes [N][K/2] u8, box 32*kCPS B x 128 rows (out-of-range columns zero-filled)
         const cuuint64_t dims[2] = {(cuuint64_t)K / 2, (cuuint64_t)N};
         const cuuint64_t strides[1] = {(cuuint64_t)K / 2};
-        const cuuint32_t box[2] = {32 * w4::kCPS, (cuuint32_t)w4::kM}, es[2] = {1, 1};
+        const cuuint32_t box[2] = {32 * w4::kCPS, (cuuint32_t)(w4::kM * w4a16_mt(N))}, es[2] = {1, 1};
         if (enc(&tc, CU_TENSOR_MAP_DATA_TYPE_UINT8, 2, const_cast<uint8_t *>(codes), dims, strides, box, es,
                 CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
@@ -518,18 +548,28 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
         const cudaError_t e = cudaMemsetAsync(y, 0, (size_t)batch * N * sizeof(float), st);
         if (e != cudaSuccess) return e;
     }
-    dim3 grid(N / w4::kM, ksplit);
+    const int MT = w4a16_mt(N);
+    dim3 grid(N / (w4::kM * MT), ksplit);
     const uint32_t *m = static_cast<const uint32_t *>(meta);
-    auto go = [&](auto kern, int sm) {
+    auto go = [&](auto kern, int sm, int threads) {
         cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
-        kern<<<grid, w4::kThreads, sm, st>>>(tc, tx, m, packed, y, N, K, batch, ksplit);
+        kern<<<grid, threads, sm, st>>>(tc, tx, m, packed, y, N, K, batch, ksplit);
     };
-    if (BN == 64) {
-        if (packed) go(w4::w4a16_kernel<64, true>, w4::Smem<64>::BYTES);
-        else go(w4::w4a16_kernel<64, false>, w4::Smem<64>::BYTES);
+    constexpr int T1 = w4::Roles<1>::THREADS, T2 = w4::Roles<2>::THREADS;
+    if (MT == 2) {
+        if (BN == 64) {
+            if (packed) go(w4::w4a16_kernel<64, true, 2>, w4::Smem<64, 2>::BYTES, T2);
+            else go(w4::w4a16_kernel<64, false, 2>, w4::Smem<64, 2>::BYTES, T2);
+        } else {
+            if (packed) go(w4::w4a16_kernel<128, true, 2>, w4::Smem<128, 2>::BYTES, T2);
+            else go(w4::w4a16_kernel<128, false, 2>, w4::Smem<128, 2>::BYTES, T2);
+        }
+    } else if (BN == 64) {
+        if (packed) go(w4::w4a16_kernel<64, true, 1>, w4::Smem<64>::BYTES, T1);
+        else go(w4::w4a16_kernel<64, false, 1>, w4::Smem<64>::BYTES, T1);
     } else {
-        if (packed) go(w4::w4a16_kernel<128, true>, w4::Smem<128>::BYTES);
-        else go(w4::w4a16_kernel<128, false>, w4::Smem<128>::BYTES);
+        if (packed) go(w4::w4a16_kernel<128, true, 1>, w4::Smem<128>::BYTES, T1);
+        else go(w4::w4a16_kernel<128, false, 1>, w4::Smem<128>::BYTES, T1);
     }
     const cudaError_t e = cudaGetLastError();
     if (e == cudaSuccess) note_launch();

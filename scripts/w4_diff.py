@@ -13,7 +13,11 @@ for tag in ("A", "B"):
     W = (torch.randn(N, K, generator=g, device="cuda") * 0.02).half()
     c, m = lmo.lmo_quantize_groupwise(W, N, K, 1)
     x = torch.randn(B, K, generator=g, device="cuda").half()
-    res[tag] = lmo.lmo_w4a16_linear(c.view(N, K // 2), m.view(N, K // 64), N, K, x, k_split=1).cpu().numpy()
+    c, m = c.view(N, K // 2), m.view(N, K // 64)
+    if os.environ.get("PACKED") == "1":
+        res[tag] = lmo.lmo_w4a16_linear_packed(lmo.lmo_w4a16_pack(c, m, N, K), N, K, x, k_split=1).cpu().numpy()
+    else:
+        res[tag] = lmo.lmo_w4a16_linear(c, m, N, K, x, k_split=1).cpu().numpy()
 d = np.abs(res["A"] - res["B"])
 bad = d > 1e-3 * (np.abs(res["A"]) + 1e-3)
 print("max diff", d.max(), "bad elements", int(bad.sum()), "of", d.size)

@@ -256,17 +256,21 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
         const int tr = mt * kM + r;                              // row within the CTA's rows
         const uint32_t *mrow = meta + (int64_t)(n0 + tr) * (K / kK);
         const uint32_t meta_u32 = sbase + S::OFF_META + (h * kM * MT + tr) * 4;
-        auto meta_issue = [&](int j) {   // thread-private cp.async ring of the group meta words
-            if (PACKED) return;
-            if (j < nsteps) cp_async4(meta_u32 + (j % kCodes) * S::META, mrow + kb0 + j);
-            cp_commit();
+        // row-major path: the group meta word of step j is a plain read-only global load issued
+        // two steps ahead into registers (L2-resident: 1/16 of the code bytes).
+        uint32_t m_next = 0, m_next2 = 0;
+        auto meta_load = [&](int j) -> uint32_t {
+            return (!PACKED && j < nsteps) ? __ldg(mrow + kb0 + j) : 0u;
         };
-        for (int j = 0; j < kCodes - 1; ++j) meta_issue(j);
+        if (!PACKED) {
+            m_next = meta_load(0);
+            m_next2 = meta_load(1);
+        }
+        (void)meta_u32;
         const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16) + TM::A0 + mt * 32 + h * (WPT / 2);
         // software pipeline: the dequant of step j overlaps the TMEM store of step j-1
         // (tcgen05.wait::st of j-1 only after step j's arithmetic); two register buffers
         auto produce = [&](int j, uint4 (&v)[WPT / 8]) {
-            meta_issue(j + kCodes - 1);
             const int q = j / kCPS, cs = q % kCodeSlots, sub = j - q * kCPS;
             if (sub == 0) mbar_wait(&c_full[cs], (q / kCodeSlots) & 1);
             uint32_t cw[WPT / 8], mw;
@@ -286,8 +290,9 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                 asm volatile("ld.shared.u32 %0, [%1];\n"
                              : "=r"(mw) : "r"(sbase + S::OFF_CODES + cs * S::CSLOT + (mt * kCPS + sub) * S::PBLK + kM * 32 + r * 4));
             } else {
-                cp_wait<kCodes - 1>();
-                asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(meta_u32 + (j % kCodes) * S::META));
+                mw = m_next;
+                m_next = m_next2;
+                m_next2 = meta_load(j + 2);
             }
             const bool last_sub = sub == kCPS - 1 || j == nsteps - 1;
             if (!LMO_W4_WARP_ARRIVE && last_sub) mbar_arrive(&c_empty[cs]);

@@ -65,6 +65,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_NO_SCH
 #define LMO_NO_SCH 0     // 1: every schedule runs the generic kernel instance (experiments)
 #endif
+#ifndef LMO_ATTN_MINBLOCKS_GQA
+#define LMO_ATTN_MINBLOCKS_GQA 4   // 2: GQA with up to 255 registers -- faster on an 11-layer probe, slower in the 80-layer bench
+#endif
 #ifndef LMO_ATTN_MINBLOCKS
 #define LMO_ATTN_MINBLOCKS 4
 #endif
@@ -465,7 +468,8 @@ __host__ __device__ constexpr int bars_bytes() { return (NW * kStages * 8 + 127)
 // per pair, the default); 2 = pair teams with T > 1.  The specialised instances drop
 // the other modes' code (smaller kernel: fewer cold instruction-cache misses).
 template <int D, bool MHA, int NW, int SCH = 0>
-__global__ void __launch_bounds__(NW * 32, NW == kWarps ? LMO_ATTN_MINBLOCKS : 1) decode_attn_q4_kernel(const AttnArgs a) {
+__global__ void __launch_bounds__(NW * 32, NW == kWarps ? (MHA ? LMO_ATTN_MINBLOCKS : LMO_ATTN_MINBLOCKS_GQA) : 1)
+decode_attn_q4_kernel(const AttnArgs a) {
     using GG = Geo<D>;
     constexpr bool TEAMK = SCH != 0;
     constexpr int NG = GG::NG;
@@ -1585,13 +1589,13 @@ static bool sm_team_ok() {
 }
 
 template <int D>
-static int ctas_per_sm(int B_prefix) {   // (MHA and GQA variants have the same resources)
-    static int occ[64][2] = {{0}};
+static int ctas_per_sm(int B_prefix, bool mha) {   // (MHA and GQA instances differ in registers)
+    static int occ[64][2][2] = {{{0}}};
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev < 0 || dev >= 64) dev = 0;
     const int mode = B_prefix > 0 ? 1 : 0;
-    if (occ[dev][mode] == 0) {
+    if (occ[dev][mode][mha] == 0) {
         const int sz = (int)smem_bytes<D>(kMaxBatchSmem);
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kWarps, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
@@ -1599,21 +1603,38 @@ static int ctas_per_sm(int B_prefix) {   // (MHA and GQA variants have the same 
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kWarps, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
-        int n = 0, n1 = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n1, decode_attn_q4_kernel<D, true, kWarps>, kWarps * 32,
-                                                      smem_bytes<D>(mode ? kMaxBatchSmem : 0));
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, decode_attn_q4_kernel<D, false, kWarps>, kWarps * 32,
-                                                      smem_bytes<D>(mode ? kMaxBatchSmem : 0));
-        if (n1 < n) n = n1;
-        occ[dev][mode] = n > 0 ? n : 1;
+        int n = 0;
+        const size_t smem = smem_bytes<D>(mode ? kMaxBatchSmem : 0);
+        // the least occupancy over the schedule instances of this variant (same bound; SCH 0 is the largest)
+        for (int k = 0; k < 3; ++k) {
+            int m = 0;
+            if (mha)
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+                    &m, k == 0 ? decode_attn_q4_kernel<D, true, kWarps, 0> : k == 1 ? decode_attn_q4_kernel<D, true, kWarps, 1>
+                                                                            : decode_attn_q4_kernel<D, true, kWarps, 2>,
+                    kWarps * 32, smem);
+            else
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+                    &m, k == 0 ? decode_attn_q4_kernel<D, false, kWarps, 0> : k == 1 ? decode_attn_q4_kernel<D, false, kWarps, 1>
+                                                                             : decode_attn_q4_kernel<D, false, kWarps, 2>,
+                    kWarps * 32, smem);
+            if (k == 0 || m < n) n = m;
+        }
+        occ[dev][mode][mha] = n > 0 ? n : 1;
     }
-    return occ[dev][mode];
+    return occ[dev][mode][mha];
 }
 
-int attn_max_warps(int head_dim, int B_prefix) {
-    const int occ = head_dim == 64 ? ctas_per_sm<64>(B_prefix) : ctas_per_sm<128>(B_prefix);
+int attn_max_warps_v(int head_dim, int B_prefix, bool mha) {
+    const int occ = head_dim == 64 ? ctas_per_sm<64>(B_prefix, mha) : ctas_per_sm<128>(B_prefix, mha);
     return device_sm_count() * occ * kWarps;
 }
+
+int attn_max_warps(int head_dim, int B_prefix) {   // the larger of the MHA / GQA grids (scratch sizing)
+    const int a = attn_max_warps_v(head_dim, B_prefix, true), b = attn_max_warps_v(head_dim, B_prefix, false);
+    return a > b ? a : b;
+}
+
 
 size_t attn_workspace_bytes(int B, int Hkv, int Hq, int D, int num_splits) {
     const int G = Hq / Hkv;
@@ -1667,7 +1688,7 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
 
     const int D = c.head_dim;
     const int Bp = lens ? c.batch : 0;
-    const int max_ctas = attn_max_warps(D, Bp) / kWarps;
+    const int max_ctas = attn_max_warps_v(D, Bp, a.G == 1) / kWarps;
     const int64_t pairs = (int64_t)c.batch * c.kv_heads;
     const int64_t nbu = lens ? 0 : (len + kBlk - 1) / kBlk;
     a.team = 0;

@@ -169,6 +169,44 @@ def test_ties_round_half_to_even():
     assert list(codes[2:2 + len(halves)]) == [0, 2, 2, 4, 4, 14, 14]
 
 
+def test_q5_reciprocal_then_multiply_golden():
+    """Reading Q5 (Eq 10; DESIGN.md "Readings" Q5): t = RN32(RN32(x - mn) *
+    RN32(1/scale)), NOT RN32((x - mn) / scale).  Hand-computed group:
+      mn = -0.85595703125, mx = 0.93115234375 (both exact fp16), the rest 0;
+      range = 1.787109375, range/15 = 0.119140625 exactly (fp16 0x2FA0);
+      x = 0.51416015625: d = x - mn = 1.3701171875 = 1403/1024 exactly;
+      d / scale = 1403/122 = 11.5 exactly -> half-even rint -> 12 (division);
+      RN32(1/scale) = 8.393442... (rounded down), d * inv -> RN32 = 11.499999 -> 11.
+    So the oracle must emit code 11 for element 2 (a division mutation gives 12)."""
+    x = np.zeros(64)
+    x[0], x[1], x[2] = -0.85595703125, 0.93115234375, 0.51416015625
+    codes, mins, scales = quant_groups(x.astype(np.float16))
+    assert int(scales[0]) == 0x2FA0                  # 0.119140625
+    assert int(mins[0]) == 0xBAD9                    # -0.85595703125
+    assert int(codes[2]) == 11
+    assert int(codes[0]) == 0 and int(codes[1]) == 15
+
+
+def test_d1_rn32_before_rn16_golden():
+    """Reading D1 (Eq 11; DESIGN.md "Readings" D1): y = RN16(RN32(c*scale +
+    mn)).  Hand-computed group: 62 elements of 2^-24 (the min), 10.0 and 2.0.
+      range = RN32(10 - 2^-24) = 10; scale = RU16(10/15) = 683/1024 (fp16 0x3956);
+      x = 2.0: d = RN32(2 - 2^-24) = 2 (tie, even), t = 2 * RN32(1/scale) = 2.9985 -> code 3;
+      exact = 3 * 683/1024 + 2^-24 = 2 + 2^-10 + 2^-24;
+      RN32(exact) = 2 + 2^-10 (ulp32 at 2 is 2^-22) -> RN16: exact half-ulp tie -> 2.0 = 0x4000;
+      without the RN32 step the 2^-24 breaks the tie upward -> 0x4001."""
+    x = np.full(64, 2.0 ** -24)
+    x[0], x[1] = 10.0, 2.0
+    xh = x.astype(np.float16)
+    c, m = oracle.quantize_groupwise(xh, 1, 64, 1)
+    assert int(m.reshape(-1)[1]) == 0x3956
+    codes, _, _ = quant_groups(xh)
+    assert int(codes[1]) == 3 and int(codes[0]) == 15
+    y = oracle.dequantize_groupwise(c, m, 1, 64, 1).reshape(-1).view(np.uint16)
+    assert int(y[1]) == 0x4000
+    assert int(y[2]) == 0x0001                       # the min itself: code 0 -> mn exactly
+
+
 def test_pack_byte_vectors():
     """Reading 9 (low nibble = even element): codes 0..15 -> 0x10 0x32 ... 0xFE."""
     x = (np.arange(64) % 16).astype(np.float16)

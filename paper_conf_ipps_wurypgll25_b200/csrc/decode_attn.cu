@@ -368,6 +368,14 @@ __device__ __forceinline__ float fast_exp2(float x) {
     return y;
 }
 
+// floor(log2(h)) of a positive finite fp16 bit pattern (subnormals included)
+__device__ __forceinline__ int floor_log2_h(uint32_t h) {
+    const int e = (int)(h >> 10);
+    return e ? e - 15 : (31 - __clz((int)h)) - 24;
+}
+// 2^e as an fp32 (e in [-126, 127])
+__device__ __forceinline__ float exp2i(int e) { return __uint_as_float((uint32_t)(e + 127) << 23); }
+
 __device__ __forceinline__ uint32_t movmatrix_t(uint32_t x) {
     uint32_t y;
     asm("movmatrix.sync.aligned.m8n8.trans.b16 %0, %1;\n" : "=r"(y) : "r"(x));
@@ -634,6 +642,8 @@ decode_attn_q4_kernel(const AttnArgs a) {
     // every lane's C holds real scores); qs = per-group sums of q for heads 2t, 2t+1
     uint32_t qf[NG][4][2];
     float qs[NG][2];
+    const float zs = a.scale_log2;            // sigma * log2(e)
+    float zk = 0.f;                           // K-score scale of the loaded q: zs * 2^24 * 2^-Eq
     auto fetch_q = [&](int b, int kvh, uint4 (&raw)[NG][2]) {
 #pragma unroll
         for (int grp = 0; grp < NG; ++grp) {
@@ -645,7 +655,24 @@ decode_attn_q4_kernel(const AttnArgs a) {
             }
         }
     };
+    // The MMA operand is q' = q * 2^Eq (one power of two per pair, max|q'| in [2^14, 2^15)),
+    // and the 2^-20 code slots meet q'/16: without the rescale a small q (|q| < 2^-10)
+    // would become an fp16 subnormal after /16 and lose bits.  2^-Eq is folded into zk.
     auto build_q = [&](const uint4 (&raw)[NG][2]) {
+        uint32_t mx = 0;                                  // max |q| of the pair (fp16 bits)
+#pragma unroll
+        for (int grp = 0; grp < NG; ++grp)
+#pragma unroll
+            for (int k = 0; k < 2; ++k) {
+                const uint32_t w[4] = {raw[grp][k].x, raw[grp][k].y, raw[grp][k].z, raw[grp][k].w};
+#pragma unroll
+                for (int i = 0; i < 4; ++i) mx = max(mx, max(w[i] & 0x7FFFu, (w[i] >> 16) & 0x7FFFu));
+            }
+        mx = __reduce_max_sync(0xffffffffu, mx);
+        int eq = 0;
+        if (mx) eq = 14 - floor_log2_h(mx);               // in [-1, 38]
+        const float qsc = exp2i(eq);
+        zk = zs * 16777216.0f * exp2i(-eq);
 #pragma unroll
         for (int grp = 0; grp < NG; ++grp) {
             const __half *h0 = reinterpret_cast<const __half *>(&raw[grp][0]);
@@ -654,8 +681,8 @@ decode_attn_q4_kernel(const AttnArgs a) {
             float sum = 0.f;
 #pragma unroll
             for (int i = 0; i < 8; ++i) {
-                q16[i] = h0[i];
-                q16[8 + i] = h1[i];
+                q16[i] = __float2half_rn(__half2float(h0[i]) * qsc);
+                q16[8 + i] = __float2half_rn(__half2float(h1[i]) * qsc);
                 sum += __half2float(h0[i]) + __half2float(h1[i]);
             }
             sum = sum_over_t(sum);                              // Qs of head g
@@ -800,8 +827,6 @@ decode_attn_q4_kernel(const AttnArgs a) {
     constexpr int dSM = kBlk * GG::ROW;
 
     const float NEG_INF = -INFINITY;
-    const float zs = a.scale_log2;            // sigma * log2(e)
-    const float zs24 = zs * 16777216.0f;      // ... * 2^24 (K products are q c 2^-24)
     int slot = 0;                             // consumer ring position
     uint32_t phase = 0;
 #if LMO_ATTN_PROFILE
@@ -866,6 +891,42 @@ decode_attn_q4_kernel(const AttnArgs a) {
         for (int grp = 0; grp < NG; ++grp) pm[0][grp] = pm[1][grp] = 0.f;
 #pragma unroll
         for (int i = 0; i < NG * 4; ++i) acc[i][0] = acc[i][1] = acc[i][2] = acc[i][3] = 0.f;
+        // V operand exponent: the MMA's B operand is w = p' * scaleV with p' = exp2(z - mE),
+        // mE = m_run - Ei, so every w < 2^15 and the largest ones are normal fp16 (a small V
+        // scale would otherwise make p * scaleV an fp16 subnormal).  l, Pm and acc all carry
+        // the same 2^Ei, which cancels in o = (acc + Pm) / l; the partial records store mE.
+        // Ei starts at 0 with vthr = the least nonzero scale, so the first nonzero V scale
+        // sets it; afterwards it only decreases (a stage whose scale * 2^Ei >= 2^15).
+        int Ei = 0;
+        uint32_t vthr = 0x10000u;                 // V meta word >= vthr <=> scale >= 2^(15 - Ei)
+        float mE[2] = {NEG_INF, NEG_INF};
+        // rare, warp-uniform: lower Ei to fit the largest V scale vx (meta word) of the warp;
+        // returns the factor applied to l, Pm and acc (the caller rescales its live p)
+        auto v_exp = [&](uint32_t vx) -> float {
+            const int fl = floor_log2_h(__reduce_max_sync(0xffffffffu, vx >> 16));
+            const int En = 14 - fl;
+            const float f = exp2i(En - Ei);
+            Ei = En;
+            const int k = fl + 1;                 // new threshold 2^k
+            vthr = (k >= -14 ? (uint32_t)(k + 15) << 10 : 1u << (k + 24)) << 16;
+            l_run[0] *= f;
+            l_run[1] *= f;
+#pragma unroll
+            for (int grp = 0; grp < NG; ++grp) {
+                pm[0][grp] *= f;
+                pm[1][grp] *= f;
+            }
+#pragma unroll
+            for (int i = 0; i < NG * 4; ++i) {
+                acc[i][0] *= f;
+                acc[i][1] *= f;
+                acc[i][2] *= f;
+                acc[i][3] *= f;
+            }
+            mE[0] = m_run[0] - (float)Ei;
+            mE[1] = m_run[1] - (float)Ei;
+            return f;
+        };
 
         // K part of one stage (ring position sl/ph): wait for the data, scores
         auto wait_stage = [&](int sl, uint32_t ph) {
@@ -921,7 +982,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
 #pragma unroll
                 for (int grp = 0; grp < NG; ++grp) {
                     const float2 f = meta_f2(grp == 0 ? km.x : km.y);
-                    z = fmaf(S[grp], f.y * zs24, fmaf(f.x * zs, qs[grp][0], z));
+                    z = fmaf(S[grp], f.y * zk, fmaf(f.x * zs, qs[grp][0], z));
                 }
                 const int tokbase = (blk0 + jb + ls) * kBlk;
                 if (M == 0 && (ls >= nsub || tokbase + row >= L)) z = NEG_INF;
@@ -956,7 +1017,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
 #pragma unroll
                         for (int grp = 0; grp < NG; ++grp) {
                             const float2 f = meta_f2(grp == 0 ? km.x : km.y);
-                            const float sk = f.y * zs24;
+                            const float sk = f.y * zk;
                             const float mk = f.x * zs;
                             z0 = fmaf(sacc[grp][2 * r + 0], sk, fmaf(mk, qs[grp][0], z0));
                             z1 = fmaf(sacc[grp][2 * r + 1], sk, fmaf(mk, qs[grp][1], z1));
@@ -1001,6 +1062,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
                 if (mb > m_run[0]) {                          // warp-uniform
                     const float a0 = fast_exp2(m_run[0] - mb);
                     m_run[0] = mb;
+                    mE[0] = mb - (float)Ei;
                     l_run[0] *= a0;
 #pragma unroll
                     for (int grp = 0; grp < NG; ++grp) pm[0][grp] *= a0;
@@ -1013,9 +1075,14 @@ decode_attn_q4_kernel(const AttnArgs a) {
                     }
                 }
                 }
-                const float p = fast_exp2(z - m_run[0]);
-                l_run[0] += p;
+                float p = fast_exp2(z - mE[0]);
                 const uint2 vmw = load_meta<NG>(ring_u32 + st + ls * dSM + row * GG::ROW + GG::OVM);
+                {
+                    uint32_t vx = NG == 2 ? max(vmw.x, vmw.y) : vmw.x;
+                    if (M != 1 && z == NEG_INF) vx = 0u;                  // stale meta of masked slots
+                    if (__any_sync(0xffffffffu, vx >= vthr)) p *= v_exp(vx);
+                }
+                l_run[0] += p;
                 float w[2] = {0.f, 0.f};
 #pragma unroll
                 for (int grp = 0; grp < NG; ++grp) {
@@ -1073,6 +1140,8 @@ decode_attn_q4_kernel(const AttnArgs a) {
                 const float a0 = fast_exp2(m_run[0] - mn0), a1 = fast_exp2(m_run[1] - mn1);
                 m_run[0] = mn0;
                 m_run[1] = mn1;
+                mE[0] = mn0 - (float)Ei;
+                mE[1] = mn1 - (float)Ei;
                 l_run[0] *= a0;
                 l_run[1] *= a1;
 #pragma unroll
@@ -1095,15 +1164,31 @@ decode_attn_q4_kernel(const AttnArgs a) {
                     float p[2][2];
 #pragma unroll
                     for (int r = 0; r < 2; ++r) {
-                        p[r][0] = fast_exp2(ks.z[s][r][0] - m_run[0]);
-                        p[r][1] = fast_exp2(ks.z[s][r][1] - m_run[1]);
+                        p[r][0] = fast_exp2(ks.z[s][r][0] - mE[0]);
+                        p[r][1] = fast_exp2(ks.z[s][r][1] - mE[1]);
                     }
-                    l_run[0] += p[0][0] + p[1][0];
-                    l_run[1] += p[0][1] + p[1][1];
                     const uint32_t ss = st + s * dSC;
                     const uint32_t sm = st + s * dSM;
                     const uint2 vmA = load_meta<NG>(sm + offVm0);
                     const uint2 vmB = load_meta<NG>(sm + offVm0 + dM1);
+                    {
+                        uint32_t vxA = NG == 2 ? max(vmA.x, vmA.y) : vmA.x;
+                        uint32_t vxB = NG == 2 ? max(vmB.x, vmB.y) : vmB.x;
+                        if (tail) {                    // masked tail tokens: meta may be stale
+                            if (ks.z[s][0][0] == NEG_INF) vxA = 0u;
+                            if (ks.z[s][1][0] == NEG_INF) vxB = 0u;
+                        }
+                        const uint32_t vx = max(vxA, vxB);
+                        if (__any_sync(0xffffffffu, vx >= vthr)) {
+                            const float f = v_exp(vx);
+                            p[0][0] *= f;
+                            p[0][1] *= f;
+                            p[1][0] *= f;
+                            p[1][1] *= f;
+                        }
+                    }
+                    l_run[0] += p[0][0] + p[1][0];
+                    l_run[1] += p[0][1] + p[1][1];
 #pragma unroll
                     for (int grp = 0; grp < NG; ++grp) {
                         float2 f0 = meta_f2(grp == 0 ? vmA.x : vmA.y);
@@ -1270,7 +1355,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
                         __stcg(r4 + 1, make_float4(vo[e][grp][4], vo[e][grp][5], vo[e][grp][6], vo[e][grp][7]));
                     }
                     if (g == 0) {
-                        __stcg(rec + h * GG::REC + D, m_run[e]);
+                        __stcg(rec + h * GG::REC + D, mE[e]);
                         __stcg(rec + h * GG::REC + D + 1, lt[e]);
                     }
                 }
@@ -1363,7 +1448,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
                         __stcg(r4 + 1, make_float4(vo[e][grp][4], vo[e][grp][5], vo[e][grp][6], vo[e][grp][7]));
                     }
                     if (g == 0) {
-                        __stcg(rec + h * GG::REC + D, m_run[e]);
+                        __stcg(rec + h * GG::REC + D, mE[e]);
                         __stcg(rec + h * GG::REC + D + 1, lt[e]);
                     }
                 }

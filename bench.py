@@ -3,16 +3,22 @@
 
 A "step" is one decode step of the whole hot path over all layers of the
 workload: for every layer, append-quantize the new token's K/V (A2) and run
-decode attention over the q4 cache (A3+A4).  Inputs are seeded synthetic
-tensors shaped like the paper's OPT/LLaMA workloads, resident in HBM before
-the timed region (value) or copied from pinned host memory inside it (e2e).
+decode attention over the q4 cache (A3+A4), one fused launch per layer
+(lmo_decode_step_q4).  Inputs are seeded synthetic tensors shaped like the
+paper's OPT/LLaMA workloads, resident in HBM before the timed region (value)
+or copied from pinned host memory inside it (e2e).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2] [--impl ours|reference]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config c4]
+                  [--scaling strong|weak] [--impl ours|reference]
 
-Multi-GPU (torchrun, one rank per GPU, NCCL): the batch is sharded by
-sequence -- weak scaling, each rank owns a full config-sized batch at its own
-global batch offset; no collective in the hot path (timing reduce only).
-Prints ONE JSON line on rank 0.
+Default workload: c4 (OPT-66B-shaped), the largest BASELINE.json config that
+fits one GPU (c5 is the 8-GPU config).  Multi-GPU (torchrun, one rank per
+GPU, NCCL): the batch is sharded by sequence -- strong scaling by default (the
+config's global batch split over the ranks, BASELINE.json north star), weak
+scaling with --scaling weak; no collective in the hot path.  After the timed
+region the sampled outputs of every rank are gathered to rank 0 (NCCL
+all_gather, C1) and checked against the CPU oracle.  Prints ONE JSON line on
+rank 0.
 """
 from __future__ import annotations
 
@@ -32,7 +38,9 @@ from paper_conf_ipps_wurypgll25_b200 import configs as C  # noqa: E402
 from paper_conf_ipps_wurypgll25_b200 import inputs as I  # noqa: E402
 
 METRIC = "q4-KV decode-attention tokens/s & achieved HBM GB/s at 1/2/4/8 B200"
-FALLBACK_HBM = 6650.0
+FALLBACK_HBM = 6650.0      # B200_PROFILING.md fallback copy bandwidth (GB/s)
+NOMINAL_HBM = 8000.0       # B200 HBM3e nominal (the north star's "about 8 TB/s")
+TOL = 2e-3                 # BASELINE.json north star attention bar (normwise, reading 17)
 
 
 def parse():
@@ -40,33 +48,36 @@ def parse():
     p.add_argument("--gpus", type=int, default=1)
     p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=3)
-    p.add_argument("--config", default="c2", choices=sorted(C.CONFIGS))
+    p.add_argument("--config", default="c4", choices=sorted(C.CONFIGS))
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--splits", type=int, default=0, help="num_splits (0 = stream-K auto)")
+    p.add_argument("--scaling", default="strong", choices=["strong", "weak"])
+    p.add_argument("--splits", type=int, default=0, help="num_splits (0 = library auto)")
+    p.add_argument("--verify-pairs", type=int, default=4, help="C1 sampled (layer, b, kv-head) per rank")
     p.add_argument("--no-e2e", action="store_true")
-    p.add_argument("--no-stream", action="store_true", help="skip the A1/A5 weight streaming leg")
+    p.add_argument("--no-stream", action="store_true", help="skip the A1/A5 weight streaming and W4A16 legs")
     p.add_argument("--no-offload", action="store_true", help="skip the host-offloaded KV leg")
     p.add_argument("--no-early", action="store_true", help="disable LMO_STEP_CACHE_STABLE")
-    p.add_argument("--cpu-sample-seconds", type=float, default=10.0)
+    p.add_argument("--cpu-sample-seconds", type=float, default=10.0,
+                   help="oracle baseline: CPU seconds on all cores (single core: half of it)")
     return p.parse_args()
 
 
-def peaks():
+def copy_peak():
     path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     try:
         d = json.load(open(path))
-        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy read+write)"
     except Exception:
         return FALLBACK_HBM, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def workload_config(w: C.Workload, n: int, extra=None):
+def workload_config(w: C.Workload, world: int, sh, mode: str, extra=None):
     d = {
         "workload": f"{w.key}: {w.name}",
-        "batch_per_gpu": w.batch, "global_batch": w.batch * n, "q_heads": w.q_heads,
+        "global_batch": sh.global_batch, "batch_per_gpu": sh.batch, "q_heads": w.q_heads,
         "kv_heads": w.kv_heads, "head_dim": w.head_dim, "layers": w.layers,
         "prompt": w.prompt, "gen": w.gen, "kv_format": "4-bit group-wise min/scale, G=64",
-        "parallelism": f"batch-sharded dp{n} (weak scaling)",
+        "parallelism": f"batch-sharded dp{world} ({mode} scaling)",
     }
     if extra:
         d.update(extra)
@@ -129,71 +140,130 @@ class ClockSampler:
 
 # -------------------------------------------------------- CPU oracle -------
 
-def cpu_oracle_rate(w: C.Workload, target_s: float, nthreads: int):
-    """Time the oracle (as it stands) on a bounded sample of decode work at the
-    mean decode length: whole layers' worth of (sequence, kv-head) pairs (one
-    append + one attention each), repeated over layers until ~target_s of CPU
-    wall time; extrapolated linearly to tokens/s of the whole workload."""
-    import numpy as np
-    import oracle
-    seed = I.seed_for_config(w.index)
-    L = w.prompt + w.gen // 2
-    d, G = w.head_dim, w.group_ratio
-    pairs_total = w.batch * w.kv_heads
-    units = [(l, b, h) for l in range(w.layers) for b in range(w.batch) for h in range(w.kv_heads)]
-    done, elapsed, npairs = 0, 0.0, max(1, nthreads)
-    while elapsed < target_s and done < len(units):
-        chunk = units[done:done + npairs]
-        B = len(chunk)
-        cache = oracle.new_cache(B, 1, L + 1, d)
-        ks = np.stack([I.gen_f16(seed, I.STREAM_K, l, b, 1, h, 1, 0, L + 1, d)[0] for l, b, h in chunk])
-        vs = np.stack([I.gen_f16(seed, I.STREAM_V, l, b, 1, h, 1, 0, L + 1, d)[0] for l, b, h in chunk])
-        qs = np.stack([I.gen_f16(seed, I.STREAM_Q, l, b, 1, h * G, G, 0, 1, d, group=G)[0, :, 0]
-                       for l, b, h in chunk])
-        oracle.kv_append_quant(cache, ks[:, :, :L], vs[:, :, :L], 0)   # resident cache (untimed)
+class OracleSample:
+    """A bounded sample of one decode step's work for the CPU oracle (as it stands):
+    `n_units` distinct (layer, sequence, kv-head) units of the workload at the mean
+    decode length L = s + n/2, each with its cache of L-1 old tokens prefilled ONCE
+    (untimed, like the resident cache of a real decode).  One pass = per unit the
+    append-quantize of the new token at slot L-1 (A2) and attention of its G query
+    heads over L tokens (A3) -- exactly one decode step's work for those units.  The
+    work of a step is linear in units, so a pass extrapolates to the full step by
+    (B * Hkv * layers) / n_units."""
+
+    def __init__(self, w: C.Workload, n_units: int):
+        import numpy as np
+        import oracle
+        self.w = w
+        seed = I.seed_for_config(w.index)
+        self.L = w.prompt + w.gen // 2
+        d, G, L = w.head_dim, w.group_ratio, self.L
+        total = w.layers * w.batch * w.kv_heads
+        n_units = max(1, min(n_units, total))
+        stride = max(1, total // n_units)          # units spread over the whole step
+        units = []
+        for j in range(n_units):
+            x = (j * stride) % total
+            l, r = divmod(x, w.batch * w.kv_heads)
+            units.append((l, *divmod(r, w.kv_heads)))
+        self.units = units
+        self.cache = oracle.new_cache(len(units), 1, L, d)
+        ks = np.stack([I.gen_f16(seed, I.STREAM_K, l, b, 1, h, 1, 0, L, d)[0] for l, b, h in units])
+        vs = np.stack([I.gen_f16(seed, I.STREAM_V, l, b, 1, h, 1, 0, L, d)[0] for l, b, h in units])
+        self.q = np.ascontiguousarray(np.stack(
+            [I.gen_f16(seed, I.STREAM_Q, l, b, 1, h * G, G, L - w.prompt - 1, 1, d, group=G)[0, :, 0]
+             for l, b, h in units]))
+        oracle.kv_append_quant(self.cache, ks[:, :, :L - 1], vs[:, :, :L - 1], 0)   # resident (untimed)
+        self.k_new = np.ascontiguousarray(ks[:, :, L - 1:])
+        self.v_new = np.ascontiguousarray(vs[:, :, L - 1:])
+        self.units_per_step = total
+
+    def run(self, nthreads: int) -> float:
+        """One timed pass (A2 append + A3 attention of every unit); seconds."""
+        import oracle
         t0 = time.perf_counter()
-        oracle.kv_append_quant(cache, ks[:, :, L:], vs[:, :, L:], L)    # A2 (timed)
-        oracle.decode_attention_q4(cache, qs, L + 1, nthreads=nthreads)  # A3 (timed)
-        elapsed += time.perf_counter() - t0
-        done += B
-        npairs = min(len(units) - done, npairs * 2)
-    t_unit = elapsed / done
-    t_step = t_unit * pairs_total * w.layers
-    tokens_per_s = w.batch / t_step
-    by = C.layer_step_bytes(w, L + 1) * w.layers
+        oracle.kv_append_quant(self.cache, self.k_new, self.v_new, self.L - 1)
+        oracle.decode_attention_q4(self.cache, self.q, self.L, nthreads=nthreads)
+        return time.perf_counter() - t0
+
+    def tokens_per_s(self, seconds_per_pass: float) -> float:
+        t_step = seconds_per_pass * self.units_per_step / len(self.units)
+        return self.w.batch / t_step
+
+
+def oracle_rate(w: C.Workload, target_s: float, nthreads: int, cpus=None):
+    """Time the oracle on `nthreads` threads (optionally pinned to `cpus`, the
+    `taskset` equivalent) for about target_s seconds of repeated passes over one
+    bounded sample; returns the baseline dict of the bench line."""
+    old = os.sched_getaffinity(0)
+    if cpus is not None:
+        os.sched_setaffinity(0, cpus)
+    try:
+        s = OracleSample(w, max(8, 4 * nthreads))
+        s.run(nthreads)                                       # warm (page-in)
+        reps, el = 0, 0.0
+        while el < target_s and reps < 10000:
+            el += s.run(nthreads)
+            reps += 1
+        per = el / reps
+    finally:
+        os.sched_setaffinity(0, old)
+    L = s.L
     return {
-        "value": tokens_per_s, "unit": "tokens/s", "cores": nthreads, "kind": "oracle",
-        "sample": (f"{done} (layer, sequence, kv-head) units of one decode step at L={L + 1} "
-                   f"(append + attention of {G} q head(s) each) = {elapsed:.1f} s CPU wall on "
-                   f"{nthreads} threads; extrapolated x{pairs_total * w.layers / done:.1f} to the "
-                   f"{pairs_total} x {w.layers} units of a step (work is linear in units)"),
-        "gbs_equiv": by / t_step / 1e9,
+        "value": s.tokens_per_s(per), "unit": "tokens/s", "cores": nthreads, "kind": "oracle",
+        "sample": (f"{len(s.units)} (layer, sequence, kv-head) units of one decode step at L={L} "
+                   f"(A2 append of the new token + A3 attention of {w.group_ratio} q head(s) each), "
+                   f"caches prefilled untimed; {reps} timed passes = {el:.1f} s wall on {nthreads} "
+                   f"thread(s){' pinned to cpu ' + ','.join(map(str, sorted(cpus))) if cpus else ''}; "
+                   f"extrapolated x{s.units_per_step / len(s.units):.0f} to the {s.units_per_step} units "
+                   f"of a step (work is linear in units)"),
+        "ms_per_step": 1e3 * w.batch / s.tokens_per_s(per),
     }
 
 
+def cpu_baselines(w: C.Workload, target_s: float):
+    allc = sorted(os.sched_getaffinity(0))
+    multi = oracle_rate(w, target_s, len(allc))
+    single = oracle_rate(w, max(1.0, target_s / 2), 1, cpus={allc[0]})
+    multi.pop("ms_per_step", None)
+    single.pop("ms_per_step", None)
+    multi["single_core"] = single
+    return multi
+
+
 def run_reference(args):
+    """The base contract's reference arm = the oracle as it stands on the host cores:
+    each step is one bounded sample pass (sized to ~2 s), warm-up steps untimed."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
     w = C.CONFIGS[args.config]
     nthreads = len(os.sched_getaffinity(0))
-    vals = []
-    base = None
-    per = max(1.0, min(3.0, args.cpu_sample_seconds / 3))
-    for i in range(args.warmup + args.steps):
-        r = cpu_oracle_rate(w, per if i >= args.warmup else 0.5, nthreads)
-        if i >= args.warmup:
-            vals.append(r["value"])
-            base = r
-    v = statistics.median(vals)
+    probe = OracleSample(w, max(8, 4 * nthreads))
+    t1 = min(probe.run(nthreads) for _ in range(6)) / len(probe.units)   # seconds per unit, all cores
+    n_units = int(min(w.layers * w.batch * w.kv_heads, max(2 * nthreads, 2.0 / max(t1, 1e-6))))
+    s = OracleSample(w, min(n_units, 64 * nthreads))
+    reps = max(1, int(round(n_units / len(s.units))))          # repeat the resident sample
+    for _ in range(args.warmup):
+        s.run(nthreads)
+    el = 0.0
+    for _ in range(args.steps):
+        for _ in range(reps):
+            el += s.run(nthreads)
+    per = el / (args.steps * reps)
+    v = s.tokens_per_s(per)
+    from paper_conf_ipps_wurypgll25_b200.dist import Shard
+    sh = Shard(0, w.batch, w.batch)
+    sample = (f"each step = {reps} pass(es) over {len(s.units)} resident (layer, sequence, kv-head) units "
+              f"at L={s.L} (A2 append + A3 attention each, caches prefilled untimed) on {nthreads} threads; "
+              f"{args.steps} timed steps = {el:.1f} s; extrapolated x{s.units_per_step / len(s.units):.0f} to "
+              f"the {s.units_per_step} units of a decode step")
     line = {
         "impl": "reference", "metric": METRIC, "value": v, "unit": "tokens/s",
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": 1e3 * w.batch / v, "higher_is_better": True, "scaling": "weak",
+        "ms_per_step": 1e3 * w.batch / v, "higher_is_better": True, "scaling": args.scaling,
         "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded counter-based generator)",
-        "config": workload_config(w, 1),
-        "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": nthreads, "kind": "oracle",
-                         "sample": base["sample"]},
+        "config": workload_config(w, 1, sh, args.scaling),
+        "cpu_baseline": {"value": v, "unit": "tokens/s", "cores": nthreads, "kind": "oracle", "sample": sample},
         "e2e": {"value": v, "unit": "tokens/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -201,9 +271,65 @@ def run_reference(args):
 
 # ----------------------------------------------------------- our arm -------
 
+def verify_outputs(lmo, D, w, sh, out, t, nl, n_pairs, dev):
+    """C1: every rank takes n_pairs sampled (layer, sequence, kv-head) outputs of the
+    last replayed step, all ranks' samples are gathered to rank 0 over NCCL
+    (all_gather_into_tensor) and compared with the CPU oracle there.  Outside the
+    timed region."""
+    import numpy as np
+    import torch
+    G, d = w.group_ratio, w.head_dim
+    pairs = D.sample_pairs(sh, w.kv_heads, n_pairs, salt=t)
+    layers = [(j * 7919) % nl if j > 1 else (0 if j == 0 else nl - 1) for j in range(n_pairs)]
+    rows = torch.stack([out[l, b, kvh * G:(kvh + 1) * G] for (b, kvh), l in zip(pairs, layers)])
+    coords = torch.tensor([[l, sh.b_off + b, kvh] for (b, kvh), l in zip(pairs, layers)], dtype=torch.int64,
+                          device=dev)
+    rows_all = D.gather_rows(rows.float()).cpu().numpy()
+    coords_all = D.gather_rows(coords).cpu().numpy()
+    if int(os.environ.get("RANK", "0")) != 0:
+        return None
+    import oracle
+    seed = I.seed_for_config(w.index)
+    L = w.prompt + t
+    worst = 0.0
+    for (l, gb, kvh), got in zip(coords_all.tolist(), rows_all):
+        one = oracle.new_cache(1, 1, L, d)
+        oracle.kv_append_quant(one, I.gen_f16(seed, I.STREAM_K, l, gb, 1, kvh, 1, 0, L, d),
+                               I.gen_f16(seed, I.STREAM_V, l, gb, 1, kvh, 1, 0, L, d), 0)
+        q = I.gen_f16(seed, I.STREAM_Q, l, gb, 1, kvh * G, G, t - 1, 1, d, group=G)[:, :, 0]
+        ref = oracle.decode_attention_q4(one, q, L)[0]
+        err = np.max(np.abs(got - ref), axis=-1) / np.maximum(np.max(np.abs(ref), axis=-1), 1e-30)
+        worst = max(worst, float(err.max()))
+    return {"pairs": int(len(coords_all)), "ranks": int(len(coords_all) // n_pairs), "step_t": t, "L": L,
+            "max_normwise_err": worst, "tol": TOL, "pass": bool(worst <= TOL),
+            "gather": "NCCL all_gather_into_tensor (C1)" if D.dist.is_initialized() else "single rank",
+            "coords": "(layer, global sequence, kv head) per sample"}
+
+
+def read_stream_peak(lmo, torch, dev, stream, reduce_max):
+    """Measured read-only HBM stream (4 GiB, > L2), best of 5 (GB/s)."""
+    nbytes = 4 << 30
+    buf = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    buf.fill_(1)
+    sink = torch.zeros(4096, dtype=torch.int32, device=dev)
+    best = 0.0
+    with torch.cuda.stream(stream):
+        lmo.lmo_probe_read_stream(buf, sink, stream=stream)
+        for _ in range(5):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            lmo.lmo_probe_read_stream(buf, sink, stream=stream)
+            e1.record(stream)
+            e1.synchronize()
+            best = max(best, nbytes / (reduce_max(e0.elapsed_time(e1)) / 1e3) / 1e9)
+    del buf, sink
+    return best
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
+    from paper_conf_ipps_wurypgll25_b200 import dist as D
     from paper_conf_ipps_wurypgll25_b200 import lmo
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -215,9 +341,9 @@ def run_ours(args):
         dist.init_process_group("nccl", device_id=dev)
     w = C.CONFIGS[args.config]
     seed = I.seed_for_config(w.index)
-    B, Hkv, Hq, d, G, s = w.batch, w.kv_heads, w.q_heads, w.head_dim, w.group_ratio, w.prompt
-    from paper_conf_ipps_wurypgll25_b200 import dist as D
-    b_off, _ = D.shard(rank, world, B)    # global batch offset (weak scaling, no hot-path collective)
+    sh = D.shard(rank, world, w.batch, args.scaling)
+    B, b_off = sh.batch, sh.b_off
+    Hkv, Hq, d, G, s = w.kv_heads, w.q_heads, w.head_dim, w.group_ratio, w.prompt
     nl = w.layers
     steps_total = args.warmup + args.steps
     # Timed decode steps are spread evenly over the whole generation t = 1..n-1
@@ -325,6 +451,8 @@ def run_ours(args):
                 for j in range(args.warmup):
                     graphs[t_of[j]].replay()
                 torch.cuda.current_stream().synchronize()
+        barrier()                               # every rank starts the timed region together
+        with torch.cuda.stream(stream):
             ev0.record(stream)
             for j in range(args.warmup, steps_total):
                 graphs[t_of[j]].replay()
@@ -337,10 +465,22 @@ def run_ours(args):
     barrier()
     ms = reduce_max(ev0.elapsed_time(ev1))
     clocks = clk.summary()
-    tokens = world * B * args.steps
+    tokens = sh.global_batch * args.steps
     value = tokens / (ms / 1e3)
-    step_bytes = sum(C.layer_step_bytes(w, s + t_of[j], B) * nl for j in range(args.warmup, steps_total))
-    gbs = world * step_bytes / (ms / 1e3) / 1e9
+    step_bytes = sum(C.layer_step_bytes(w, s + t_of[j], sh.global_batch) * nl
+                     for j in range(args.warmup, steps_total))
+    gbs = step_bytes / (ms / 1e3) / 1e9
+
+    # ---- C1 verification (outside the timed region): the last timed step again,
+    # sampled outputs of every rank gathered to rank 0 and checked against the oracle
+    t_v = t_of[-1]
+    with torch.cuda.stream(stream):
+        graphs[t_v].replay()
+    stream.synchronize()
+    try:
+        verify = verify_outputs(lmo, D, w, sh, out, t_v, nl, args.verify_pairs, dev)
+    except Exception as ex:   # report, never hide: a failed check is a failed line
+        verify = {"pass": False, "error": str(ex)[:300]}
 
     # ---- roofline leg: attention-only launches, CUDA events on the launching stream
     reps = 5
@@ -354,8 +494,9 @@ def run_ours(args):
     a1.synchronize()
     attn_ms = reduce_max(a0.elapsed_time(a1)) / (reps * nl)
     attn_bytes = C.attention_launch_bytes(w, s + t_mid, B)
-    peak, peak_src = peaks()
+    peak, peak_src = copy_peak()
     achieved = attn_bytes / (attn_ms / 1e3) / 1e9
+    read_peak = read_stream_peak(lmo, torch, dev, stream, reduce_max)
     traffic = None
     prof = os.path.join(ROOT, "profiles", f"ncu_{w.key}.json")
     if os.path.exists(prof):
@@ -476,20 +617,23 @@ def run_ours(args):
             o1.record(stream)
         o1.synchronize()
         off_ms = reduce_max(o0.elapsed_time(o1)) / nrep
-        # raw pinned H2D bandwidth of this box (one 1 GiB copy) for the fraction
+        # pinned H2D bandwidth of this box: 4 back-to-back 1 GiB copies (best of 3 rounds)
         hb = torch.empty(1 << 30, dtype=torch.uint8).pin_memory()
         db = torch.empty(1 << 30, dtype=torch.uint8, device=dev)
         db.copy_(hb, non_blocking=True)
         torch.cuda.synchronize()
-        p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        p0.record()
-        db.copy_(hb, non_blocking=True)
-        p1.record()
-        p1.synchronize()
-        pcie = (1 << 30) / (p0.elapsed_time(p1) / 1e3) / 1e9
+        pcie = 0.0
+        for _ in range(3):
+            p0, p1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            p0.record()
+            for _ in range(4):
+                db.copy_(hb, non_blocking=True)
+            p1.record()
+            p1.synchronize()
+            pcie = max(pcie, 4 * (1 << 30) / (p0.elapsed_time(p1) / 1e3) / 1e9)
         del hb, db
         h2d_step = nl * B * Hkv * (L - 1) * lmo.row_bytes(d)
-        offload = {"value": world * B / (off_ms / 1e3), "unit": "tokens/s", "ms_per_step": off_ms,
+        offload = {"value": sh.global_batch / (off_ms / 1e3), "unit": "tokens/s", "ms_per_step": off_ms,
                    "L": L, "ring_slots": 3, "host_bytes": host_bytes,
                    "h2d_bytes_per_step": h2d_step,
                    "d2h_bytes_per_step": nl * B * Hkv * lmo.row_bytes(d),
@@ -554,13 +698,13 @@ def run_ours(args):
         e2e_ms = reduce_max(x0.elapsed_time(x1))
         e2e = {"value": tokens / (e2e_ms / 1e3), "unit": "tokens/s", "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "ms_per_step": e2e_ms / args.steps,
+               "h2d_gb_per_s_needed_to_hide": h2d / (ms / args.steps / 1e3) / 1e9,
                "path": "pinned host inputs -> H2D (copy stream, overlapped with the previous step) -> liblmo C-ABI step graph -> D2H last-layer output"}
 
     cpu = None
     if rank == 0 and world == 1:
         try:
-            cpu = cpu_oracle_rate(w, args.cpu_sample_seconds, len(os.sched_getaffinity(0)))
-            cpu.pop("gbs_equiv", None)
+            cpu = cpu_baselines(w, args.cpu_sample_seconds)
         except Exception as ex:  # never fail the bench line on the baseline leg
             cpu = {"value": None, "error": str(ex)[:200]}
 
@@ -568,19 +712,22 @@ def run_ours(args):
         line = {
             "metric": METRIC, "value": value, "unit": "tokens/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u4+f16/f32",
+            "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "u4+f16/f32",
             "data": "synthetic (seeded counter-based generator; OPT/LLaMA-shaped K/V/q)",
-            "config": workload_config(w, world, {
+            "config": workload_config(w, world, sh, args.scaling, {
                 "l2": f"inputs larger than L2: per-step q4 KV footprint "
                       f"{sum(c.nbytes() for c in caches) / 1e9:.2f} GB per GPU cycles through 126 MB L2",
                 "num_splits": args.splits,
                 "timed_decode_steps_t": timed_t, "attention_len": f"L = s + t ({w.prompt + timed_t[0]}..{w.prompt + timed_t[-1]})"}),
-            "achieved_gbs": gbs, "frac_of_peak": gbs / peak,
+            "achieved_gbs": gbs, "frac_of_peak": gbs / peak, "frac_of_nominal": gbs / NOMINAL_HBM,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "kernel": "decode_attn_q4_kernel (attention-only launches, L=s+t_mid)",
                          "peak_source": peak_src,
+                         "frac_of_nominal_8tbs": achieved / NOMINAL_HBM,
+                         "read_stream_peak": read_peak, "frac_of_read_stream_peak": achieved / read_peak,
                          "per_launch_us": attn_ms * 1e3, "algorithmic_bytes_per_launch": attn_bytes},
+            "verify": verify,
             "prefill_ms_all_layers": pre_ms,
             "streaming": streaming,
             "w4a16": w4a16,

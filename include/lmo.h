@@ -296,6 +296,14 @@ lmo_status lmo_gen_fill_f16(void *dst, int32_t nb, int32_t nh, int32_t npos, int
                             uint64_t seed, int32_t stream_id, int32_t layer, int32_t b0,
                             int32_t h0, int32_t p0, int32_t group, void *stream);
 
+/* Read-only HBM stream (measurement support for the bench's roofline
+ * denominators): reads `bytes` (a multiple of 16, >= 16)
+ * of device memory at buf with 128-bit streaming loads over a persistent
+ * grid; sink is a device buffer of >= 4 * 4 * SM-count bytes that is written
+ * only on an impossible XOR sentinel (keeps the loads live).  buf and sink
+ * 16-byte aligned. */
+lmo_status lmo_probe_read_stream(const void *buf, size_t bytes, void *sink, void *stream);
+
 /* Number of kernels this library has launched in this process. */
 uint64_t lmo_launch_count(void);
 

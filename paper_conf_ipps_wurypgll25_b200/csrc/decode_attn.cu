@@ -27,6 +27,7 @@
 //  * GQA: the query heads sharing a kv head are the MMA's head dimension, so
 //    a KV tile is read once for all of them (8 q heads per kv head cost the
 //    same HMMA count as 1).
+#include <atomic>
 #include <cstdlib>
 #include <cstring>
 #include <type_traits>
@@ -1656,31 +1657,31 @@ static size_t smem_bytes(int B_prefix) {
 constexpr int kSmWarps = 16;
 template <int D>
 static bool sm_team_ok() {
-    static int ok[64] = {0};   // 0 unknown, 1 yes, 2 no
+    static std::atomic<int> ok[64];   // 0 unknown, 1 yes, 2 no (idempotent once-per-device probe)
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev < 0 || dev >= 64) dev = 0;
-    if (ok[dev] == 0) {
+    if (ok[dev].load(std::memory_order_acquire) == 0) {
         int n = 0, n1 = 0;
         const int sz = (int)smem_bytes<D, kSmWarps>(0);
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kSmWarps>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kSmWarps>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, decode_attn_q4_kernel<D, true, kSmWarps>, kSmWarps * 32, sz);
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n1, decode_attn_q4_kernel<D, false, kSmWarps>, kSmWarps * 32, sz);
-        ok[dev] = (n >= 1 && n1 >= 1) ? 1 : 2;
+        ok[dev].store((n >= 1 && n1 >= 1) ? 1 : 2, std::memory_order_release);
         cudaGetLastError();
     }
-    return ok[dev] == 1;
+    return ok[dev].load(std::memory_order_acquire) == 1;
 }
 
 template <int D>
 static int ctas_per_sm(int B_prefix, bool mha) {   // (MHA and GQA instances differ in registers)
-    static int occ[64][2][2] = {{{0}}};
+    static std::atomic<int> occ[64][2][2];   // idempotent once-per-device occupancy probe
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev < 0 || dev >= 64) dev = 0;
     const int mode = B_prefix > 0 ? 1 : 0;
-    if (occ[dev][mode][mha] == 0) {
+    if (occ[dev][mode][mha].load(std::memory_order_acquire) == 0) {
         const int sz = (int)smem_bytes<D>(kMaxBatchSmem);
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kWarps, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
@@ -1705,9 +1706,9 @@ static int ctas_per_sm(int B_prefix, bool mha) {   // (MHA and GQA instances dif
                     kWarps * 32, smem);
             if (k == 0 || m < n) n = m;
         }
-        occ[dev][mode][mha] = n > 0 ? n : 1;
+        occ[dev][mode][mha].store(n > 0 ? n : 1, std::memory_order_release);
     }
-    return occ[dev][mode][mha];
+    return occ[dev][mode][mha].load(std::memory_order_acquire);
 }
 
 int attn_max_warps_v(int head_dim, int B_prefix, bool mha) {
@@ -1765,8 +1766,12 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     a.num_splits = num_splits;
     a.out = out;
     a.out_f16 = out_f16;
-    static int prof_launches = 0;            // profile builds: launch i records into slot i % 16
-    a.prof_slot = prof_launches++ % 16;
+#if LMO_ATTN_PROFILE
+    static std::atomic<int> prof_launches{0};   // profile builds: launch i records into slot i % 16
+    a.prof_slot = prof_launches.fetch_add(1) % 16;
+#else
+    a.prof_slot = 0;
+#endif
     const size_t counters = ((size_t)c.batch * c.kv_heads * sizeof(int) + 255) / 256 * 256;
     a.counters = static_cast<int *>(ws);
     a.partials = reinterpret_cast<float *>(static_cast<uint8_t *>(ws) + counters);
@@ -1790,22 +1795,30 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
         a.num_splits = 0;
     } else if (num_splits == 0) {
         a.team = choose_team(pairs, (int64_t)max_ctas * kWarps);
+#ifdef LMO_EXPERIMENTS
         static const char *sched = getenv("LMO_ATTN_SCHED");   // experiments: streamk | sm | team1|2|4
         if (sched && !strcmp(sched, "streamk")) a.team = 0;
         if (sched && !strcmp(sched, "sm") && sm_able) { a.team = 0; sm = true; }
         if (sched && sched[0] == 't') a.team = atoi(sched + 4);
+#endif
     }
     if (a.k_new && !a.team && (lens || a.num_splits > 0)) {
         // fixed splits, or stream-K over per-sequence lengths: append with its own kernel first
         const cudaError_t e = launch_kv_append(c, k_new, v_new, 1, len - 1, lens, st, /*pos_from_lens=*/1);
         if (e != cudaSuccess) return e;
         a.k_new = a.v_new = nullptr;
+        // the append kernel just enqueued writes slot L-1: the attention kernel must not
+        // read any stage before griddepcontrol.wait (the early prologue only holds back
+        // the append slot when it does the append itself)
+        a.early = 0;
     }
     int64_t want_warps;
     if (a.team) {
         want_warps = (int64_t)max_ctas * kWarps;          // all CTAs; idle teams exit at once
+#ifdef LMO_EXPERIMENTS
         static const char *tight = getenv("LMO_ATTN_TIGHT");   // experiments: grid = teams
         if (tight && tight[0] == '1') want_warps = pairs * a.team;
+#endif
     } else if (lens) {
         want_warps = (int64_t)max_ctas * kWarps;
     } else {
@@ -1815,8 +1828,10 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     int64_t ctas = (want_warps + kWarps - 1) / kWarps;
     if (ctas > max_ctas) ctas = max_ctas;
     if (ctas < 1) ctas = 1;
+#ifdef LMO_EXPERIMENTS
     static const char *cap_env = getenv("LMO_ATTN_MAX_CTAS");   // tuning / experiments only
     if (cap_env && atoi(cap_env) > 0 && ctas > atoi(cap_env)) ctas = atoi(cap_env);
+#endif
     const int NW = sm ? kSmWarps : kWarps;
     if (sm) ctas = device_sm_count();
     {   // the work map (uniform-length fields; per-sequence ones are completed on device)

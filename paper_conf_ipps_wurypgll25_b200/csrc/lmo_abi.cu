@@ -36,14 +36,18 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &, const void *, int, int
                                     float, int, void *, int, void *, cudaStream_t, const void *,
                                     const void *, unsigned);
 
-// Programmatic dependent launch for the hot-path kernels (LMO_PDL=0 disables).
+// Programmatic dependent launch for the hot-path kernels (always on in release
+// builds; LMO_EXPERIMENTS builds read LMO_PDL=0 to disable it for measurements).
 bool pdl_enabled() {
-    static int v = -1;
-    if (v < 0) {
+#ifdef LMO_EXPERIMENTS
+    static const int v = [] {
         const char *e = getenv("LMO_PDL");
-        v = (e && e[0] == '0') ? 0 : 1;
-    }
+        return (e && e[0] == '0') ? 0 : 1;
+    }();
     return v == 1;
+#else
+    return true;
+#endif
 }
 cudaError_t launch_gen_fill(void *, int, int, int, int, uint64_t, int, int, int, int, int, int,
                             cudaStream_t);
@@ -51,6 +55,8 @@ size_t attn_workspace_bytes(int B, int Hkv, int Hq, int D, int num_splits);
 cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *packed, const void *x, float *y,
                          int N, int K, int batch, int ksplit, cudaStream_t st);
 cudaError_t launch_w4a16_pack(const uint8_t *codes, const void *meta, uint8_t *packed, int N, int K, cudaStream_t st);
+
+cudaError_t launch_read_stream(const void *buf, size_t bytes, void *sink, cudaStream_t st);
 
 static bool aligned16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
@@ -239,6 +245,13 @@ lmo_status lmo_w4a16_linear_packed(const uint8_t *packed, int64_t N, int64_t K, 
     if (!aligned16(packed) || !aligned16(x) || !aligned16(y)) return LMO_ERR_ALIGN;
     return cuda_status(launch_w4a16(nullptr, nullptr, packed, x, y, (int)N, (int)K, batch, k_split,
                                     static_cast<cudaStream_t>(stream)));
+}
+
+lmo_status lmo_probe_read_stream(const void *buf, size_t bytes, void *sink, void *stream) {
+    if (!buf || !sink) return LMO_ERR_NULL;
+    if (bytes < 16 || bytes % 16 != 0) return LMO_ERR_SHAPE;
+    if (!aligned16(buf) || !aligned16(sink)) return LMO_ERR_ALIGN;
+    return cuda_status(launch_read_stream(buf, bytes, sink, static_cast<cudaStream_t>(stream)));
 }
 
 uint32_t lmo_version(void) { return (1u << 16) | 0u; }

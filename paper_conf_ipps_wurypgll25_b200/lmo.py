@@ -52,10 +52,14 @@ def _load():
         "lmo_w4a16_linear": [P, P, i64, i64, P, i32, P, i32, P],
         "lmo_w4a16_pack": [P, P, i64, i64, P, P],
         "lmo_w4a16_linear_packed": [P, i64, i64, P, i32, P, i32, P],
+        "lmo_probe_read_stream": [P, ctypes.c_size_t, P, P],
         "lmo_decode_step_q4": [ctypes.POINTER(lmo_kv_cache), P, P, P, i32, i32, P, ctypes.c_float,
                                i32, P, ctypes.c_int, P, ctypes.c_size_t, ctypes.c_uint32, P],
     }
+    alt = bool(os.environ.get("LMO_LIB"))
     for name, args in sig.items():
+        if alt and not hasattr(L, name):   # an older experimental build: skip symbols it lacks
+            continue
         f = getattr(L, name)
         f.argtypes = args
         f.restype = ctypes.c_int
@@ -92,7 +96,7 @@ EXPORTS = ["lmo_quantize_groupwise", "lmo_dequantize_groupwise", "lmo_kv_append_
            "lmo_gen_fill_f16", "lmo_launch_count", "lmo_version",
            "lmo_offload_ring_bytes", "lmo_offload_create", "lmo_offload_decode_step",
            "lmo_offload_destroy", "lmo_w4a16_linear", "lmo_w4a16_packed_bytes", "lmo_w4a16_pack",
-           "lmo_w4a16_linear_packed"]
+           "lmo_w4a16_linear_packed", "lmo_probe_read_stream"]
 
 
 def _check(status: int, fn: str) -> None:
@@ -248,6 +252,13 @@ def lmo_kv_append_quant(cache: KVCache, k_new: torch.Tensor, v_new: torch.Tensor
                         pos_dev: torch.Tensor | None = None, stream=None, abi=None) -> None:
     """Append-quantize k_new/v_new [B][Hkv][n_new][d] at slots pos (Eq 7)."""
     n_new = k_new.shape[2]
+    _need_cuda(k_new, v_new, pos_dev)
+    want = (cache.batch, cache.kv_heads, n_new, cache.head_dim)
+    if k_new.dtype != torch.float16 or v_new.dtype != torch.float16 or tuple(k_new.shape) != want \
+            or tuple(v_new.shape) != want:
+        raise ValueError(f"k_new/v_new must be fp16 {want}")
+    if pos_dev is not None and (pos_dev.dtype != torch.int32 or pos_dev.numel() != cache.batch):
+        raise ValueError(f"pos_dev must be int32 [{cache.batch}]")
     c = abi if abi is not None else cache.abi()
     _check(_lib.lmo_kv_append_quant(ctypes.byref(c), _ptr(k_new), _ptr(v_new), n_new, pos0,
                                     _ptr(pos_dev), _stream(stream)), "lmo_kv_append_quant")
@@ -268,6 +279,30 @@ def attention_workspace(batch: int, kv_heads: int, q_heads: int, head_dim: int,
     return torch.zeros(n, dtype=torch.uint8, device=device)
 
 
+def _check_step_args(cache: KVCache, q, out, seq_lens, workspace, k_new=None, v_new=None):
+    """Host-side shape/dtype/device checks of the tensors handed to the C ABI (the
+    library sees raw pointers; a wrong dtype or shape here would be read or written
+    out of bounds)."""
+    _need_cuda(q, out, seq_lens, workspace, k_new, v_new)
+    B, Hkv, d = cache.batch, cache.kv_heads, cache.head_dim
+    if q.dtype != torch.float16 or q.dim() != 3 or q.shape[0] != B or q.shape[2] != d or q.shape[1] % Hkv:
+        raise ValueError(f"q must be fp16 [{B}][Hq][{d}] with Hq % {Hkv} == 0, got {q.dtype} {tuple(q.shape)}")
+    if out.dtype not in (torch.float16, torch.float32) or tuple(out.shape) != tuple(q.shape):
+        raise ValueError(f"out must be fp16/fp32 {tuple(q.shape)}, got {out.dtype} {tuple(out.shape)}")
+    if seq_lens is not None and (seq_lens.dtype != torch.int32 or seq_lens.numel() != B):
+        raise ValueError(f"seq_lens must be int32 [{B}]")
+    for t in (k_new, v_new):
+        if t is not None and (t.dtype != torch.float16 or t.numel() != B * Hkv * d):
+            raise ValueError(f"k_new/v_new must be fp16 [{B}][{Hkv}](1)[{d}]")
+    for t in (q, out, workspace, k_new, v_new, seq_lens):
+        if t is not None and t.device != cache.kv.device:
+            raise ValueError("all tensors must live on the cache's device")
+
+
+def _nbytes(t: torch.Tensor) -> int:
+    return t.numel() * t.element_size()
+
+
 def lmo_decode_attention_q4(cache: KVCache, q: torch.Tensor, length: int = 0,
                             seq_lens: torch.Tensor | None = None, softmax_scale: float | None = None,
                             num_splits: int = 0, out: torch.Tensor | None = None,
@@ -283,11 +318,12 @@ def lmo_decode_attention_q4(cache: KVCache, q: torch.Tensor, length: int = 0,
     if workspace is None:
         workspace = attention_workspace(cache.batch, cache.kv_heads, Hq, cache.head_dim,
                                         num_splits, q.device)
+    _check_step_args(cache, q, out, seq_lens, workspace)
     dt = LMO_F16 if out.dtype == torch.float16 else LMO_F32
     c = abi if abi is not None else cache.abi()
     _check(_lib.lmo_decode_attention_q4(ctypes.byref(c), _ptr(q), Hq, length, _ptr(seq_lens),
                                         float(softmax_scale), num_splits, _ptr(out), dt,
-                                        _ptr(workspace), workspace.numel(), _stream(stream)),
+                                        _ptr(workspace), _nbytes(workspace), _stream(stream)),
            "lmo_decode_attention_q4")
     return out
 
@@ -309,11 +345,12 @@ def lmo_decode_step_q4(cache: KVCache, k_new: torch.Tensor, v_new: torch.Tensor,
     if workspace is None:
         workspace = attention_workspace(cache.batch, cache.kv_heads, Hq, cache.head_dim,
                                         num_splits, q.device)
+    _check_step_args(cache, q, out, seq_lens, workspace, k_new, v_new)
     dt = LMO_F16 if out.dtype == torch.float16 else LMO_F32
     c = abi if abi is not None else cache.abi()
     _check(_lib.lmo_decode_step_q4(ctypes.byref(c), _ptr(k_new), _ptr(v_new), _ptr(q), Hq, length,
                                    _ptr(seq_lens), float(softmax_scale), num_splits, _ptr(out), dt,
-                                   _ptr(workspace), workspace.numel(), int(flags), _stream(stream)),
+                                   _ptr(workspace), _nbytes(workspace), int(flags), _stream(stream)),
            "lmo_decode_step_q4")
     return out
 
@@ -326,6 +363,13 @@ def lmo_gen_fill_f16(dst: torch.Tensor, seed: int, stream_id: int, layer: int, b
     _check(_lib.lmo_gen_fill_f16(_ptr(dst), nb, nh, npos, dim, seed, stream_id, layer, b0, h0, p0,
                                  group, _stream(stream)), "lmo_gen_fill_f16")
     return dst
+
+
+def lmo_probe_read_stream(buf: torch.Tensor, sink: torch.Tensor, stream=None) -> None:
+    """Measurement support: one read-only streaming pass over buf (bench roofline)."""
+    _need_cuda(buf, sink)
+    _check(_lib.lmo_probe_read_stream(_ptr(buf), buf.numel() * buf.element_size() // 16 * 16, _ptr(sink),
+                                      _stream(stream)), "lmo_probe_read_stream")
 
 
 # ------------------------------------------------------- NEXT-4: offloaded KV
@@ -379,7 +423,7 @@ class OffloadKV:
         dt = LMO_F16 if out.dtype == torch.float16 else LMO_F32
         _check(_lib.lmo_offload_decode_step(self._h, _ptr(k_new), _ptr(v_new), _ptr(q), Hq, length,
                                             float(softmax_scale), num_splits, _ptr(out), dt,
-                                            _ptr(workspace), workspace.numel(), _stream(stream)),
+                                            _ptr(workspace), _nbytes(workspace), _stream(stream)),
                "lmo_offload_decode_step")
         return out
 

@@ -1,4 +1,10 @@
-"""World-size-2 gloo tests of the sharded (batch-split, collective-free) host logic."""
+"""World-size-2 gloo tests of the sharded (batch-split, collective-free) host logic
+(SURVEY §8(e)): shard bounds in both scaling modes, generator slicing, the C1
+verification gather (the bench's own `verify_outputs`) and the C2 timing reduce.
+
+The per-rank compute is the CPU oracle here (no GPU in this container): two
+strong-scaling shards of one batch, each computed on its own rank and gathered,
+must reproduce the unsharded computation exactly."""
 import os
 import socket
 
@@ -10,6 +16,7 @@ import torch.multiprocessing as mp
 
 from paper_conf_ipps_wurypgll25_b200 import dist as D
 from paper_conf_ipps_wurypgll25_b200 import inputs as I
+from paper_conf_ipps_wurypgll25_b200.configs import CONFIGS
 
 
 def _free_port():
@@ -20,26 +27,54 @@ def _free_port():
     return p
 
 
+def oracle_layer_out(w, layer, b_off, B, t):
+    """Oracle outputs [B][Hq][d] of one layer at decode step t for global sequences
+    [b_off, b_off + B) (generator at global coordinates)."""
+    import oracle
+    seed = I.seed_for_config(w.index)
+    L, d, G = w.prompt + t, w.head_dim, w.group_ratio
+    cache = oracle.new_cache(B, w.kv_heads, L, d)
+    oracle.kv_append_quant(cache, I.gen_f16(seed, I.STREAM_K, layer, b_off, B, 0, w.kv_heads, 0, L, d),
+                           I.gen_f16(seed, I.STREAM_V, layer, b_off, B, 0, w.kv_heads, 0, L, d), 0)
+    q = I.gen_f16(seed, I.STREAM_Q, layer, b_off, B, 0, w.q_heads, t - 1, 1, d, group=G)[:, :, 0]
+    return oracle.decode_attention_q4(cache, q, L, nthreads=2)
+
+
 def _worker(rank, world, port, q):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank),
                       WORLD_SIZE=str(world))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
-        B = 3
-        b_off, gB = D.shard(rank, world, B)
-        # a rank's slice of the seeded inputs == the same rows of the global batch
-        kv = I.gen_f16(I.seed_for_config(4), I.STREAM_K, 5, b_off, B, 0, 2, 100, 4, 128)
+        res = {}
+        # weak: a rank's slice of the seeded inputs == the same rows of the global batch
+        sh = D.shard(rank, world, 3, "weak")
+        kv = I.gen_f16(I.seed_for_config(4), I.STREAM_K, 5, sh.b_off, sh.batch, 0, 2, 100, 4, 128)
         allk = D.gather_rows(torch.from_numpy(kv.astype(np.float32))).numpy().astype(np.float16)
-        ref = I.gen_f16(I.seed_for_config(4), I.STREAM_K, 5, 0, gB, 0, 2, 100, 4, 128)
-        ok_gen = np.array_equal(allk, ref)
-        # timing reduce returns the slowest rank's time on every rank
-        t = D.max_over_ranks(1.5 + rank)
-        q.put((rank, ok_gen, t, gB))
+        ref = I.gen_f16(I.seed_for_config(4), I.STREAM_K, 5, 0, sh.global_batch, 0, 2, 100, 4, 128)
+        res["gen_weak"] = np.array_equal(allk, ref)
+        # strong: c1's batch (4 sequences) split 2 + 2; each rank computes its shard's
+        # outputs; gathered, they equal the unsharded batch's outputs bit for bit
+        w = CONFIGS["c1"]
+        sh = D.shard(rank, world, w.batch, "strong")
+        t = w.steps
+        mine = oracle_layer_out(w, 0, sh.b_off, sh.batch, t)
+        allo = D.gather_rows(torch.from_numpy(mine)).numpy()
+        full = oracle_layer_out(w, 0, 0, w.batch, t)
+        res["strong_gather_equals_unsharded"] = np.array_equal(allo, full)
+        # the bench's C1 verification path (sampling, coordinates, gather, oracle check)
+        # on a shard "result" that is the oracle's own output (as fp32): must pass, error ~1e-8
+        import bench
+        out = torch.from_numpy(mine[None].astype(np.float32))             # [layers=1][B][Hq][d]
+        v = bench.verify_outputs(None, D, w, sh, out, t, 1, 3, torch.device("cpu"))
+        res["verify"] = v
+        # C2: the timing reduce returns the slowest rank's time on every rank
+        res["max"] = D.max_over_ranks(1.5 + rank)
+        q.put((rank, res))
     finally:
         dist.destroy_process_group()
 
 
-def test_two_rank_sharding_and_timing_reduce():
+def test_two_rank_sharding_gather_verify_and_timing_reduce():
     world = 2
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -47,17 +82,43 @@ def test_two_rank_sharding_and_timing_reduce():
     procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
     for p in procs:
         p.start()
-    res = sorted(q.get(timeout=120) for _ in range(world))
+    res = dict(q.get(timeout=300) for _ in range(world))
     for p in procs:
         p.join(timeout=60)
-    assert all(r[1] for r in res)
-    assert all(r[2] == 2.5 for r in res)
-    assert all(r[3] == 6 for r in res)
+    for r in range(world):
+        assert res[r]["gen_weak"]
+        assert res[r]["strong_gather_equals_unsharded"]
+        assert res[r]["max"] == 2.5
+    v = res[0]["verify"]
+    assert v["pass"] and v["pairs"] == 6 and v["ranks"] == 2 and v["max_normwise_err"] < 1e-6   # fp32 rows
+    assert res[1]["verify"] is None                    # only rank 0 checks
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
+@pytest.mark.parametrize("batch", [8, 64, 128, 13])
+def test_strong_shards_partition_the_batch(world, batch):
+    """Strong scaling: contiguous, non-empty, near-equal shards covering [0, B) once."""
+    shards = [D.shard(r, world, batch, "strong") for r in range(world)]
+    assert shards[0].b_off == 0
+    for a, b in zip(shards, shards[1:]):
+        assert b.b_off == a.b_off + a.batch
+    assert shards[-1].b_off + shards[-1].batch == batch
+    assert all(s.global_batch == batch for s in shards)
+    sizes = [s.batch for s in shards]
+    assert min(sizes) >= 1 and max(sizes) - min(sizes) <= 1
 
 
 def test_shard_bounds():
-    assert D.shard(0, 1, 32) == (0, 32)
-    assert D.shard(7, 8, 16) == (112, 128)
+    assert D.shard(0, 1, 32, "weak") == D.Shard(0, 32, 32)
+    assert D.shard(7, 8, 16, "weak") == D.Shard(112, 16, 128)
+    assert D.shard(7, 8, 128, "strong") == D.Shard(112, 16, 128)      # c5: 128 over 8 -> 16 per GPU
     with pytest.raises(ValueError):
         D.shard(2, 2, 4)
+    with pytest.raises(ValueError):
+        D.shard(0, 8, 4, "strong")                                     # c1 (B=4) supports <= 4 GPUs
+    with pytest.raises(ValueError):
+        D.shard(0, 2, 4, "diagonal")
     assert D.max_over_ranks(3.0) == 3.0
+    pairs = D.sample_pairs(D.shard(1, 2, 64, "strong"), 72, 5)
+    assert len(pairs) == 5 and pairs[0] == (0, 0) and pairs[1] == (31, 71)
+    assert all(0 <= b < 32 and 0 <= h < 72 for b, h in pairs)

@@ -588,3 +588,35 @@ def test_decode_loop_cache_stable_chain(lmo):
             ref = oracle.decode_attention_q4(host, q[l, t].view(B, H, d).cpu().numpy(), s0 + t + 1,
                                              nthreads=8)
             check_attention(res[(l, t)].cpu().numpy(), ref, f"cache-stable chain layer {l} step {t}")
+
+
+# ------------------------------------------------ §8(e): sharding invariance --
+
+@pytest.mark.parametrize("G,d", [(1, 128), (8, 128), (2, 64)])
+def test_sharded_step_bit_identical(lmo, G, d):
+    """Batch sharding: the fused step on the two halves of a batch --
+    each half its own cache, inputs generated at the global coordinates, as two ranks
+    hold them -- is bit-identical to one full-batch call when the team size is fixed
+    (num_splits=1: one warp per (sequence, kv head) pair, no cross-pair state)."""
+    B, Hkv, L, seed = 8, 3, 211, 4242
+    Hq = Hkv * G
+
+    def run(b0, nb):
+        cache = lmo.KVCache.empty(nb, Hkv, L, d)
+        kf = torch.empty((nb, Hkv, L, d), dtype=torch.float16, device="cuda")
+        vf = torch.empty_like(kf)
+        lmo.lmo_gen_fill_f16(kf, seed, I.STREAM_K, 0, b0, 0, 0)
+        lmo.lmo_gen_fill_f16(vf, seed, I.STREAM_V, 0, b0, 0, 0)
+        lmo.lmo_kv_append_quant(cache, kf[:, :, :L - 1].contiguous(), vf[:, :, :L - 1].contiguous(), pos0=0)
+        q = torch.empty((nb, Hq, 1, d), dtype=torch.float16, device="cuda")
+        lmo.lmo_gen_fill_f16(q, seed, I.STREAM_Q, 0, b0, 0, 0, group=G)
+        out = lmo.lmo_decode_step_q4(cache, kf[:, :, L - 1].contiguous(), vf[:, :, L - 1].contiguous(),
+                                     q.view(nb, Hq, d), L, num_splits=1, flags=lmo.LMO_STEP_CACHE_STABLE)
+        torch.cuda.synchronize()
+        return out.cpu(), cache.kv[:, :, :L].cpu()        # slots >= L: never written
+
+    full, kv_full = run(0, B)
+    lo, kv_lo = run(0, B // 2)
+    hi, kv_hi = run(B // 2, B // 2)
+    assert torch.equal(torch.cat([lo, hi]), full)
+    assert torch.equal(torch.cat([kv_lo, kv_hi]), kv_full)

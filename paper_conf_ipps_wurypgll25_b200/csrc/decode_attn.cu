@@ -838,7 +838,12 @@ decode_attn_q4_kernel(const AttnArgs a) {
 #endif
     int team_k = 0;                           // pairs finished (team mode: scratch double buffer)
 
-    while (!ctl.cc.done) {
+    for (;;) {
+        {   // every lane reads the flag before lane 0 advances the iterator (WAR on ctl.cc)
+            const bool all_done = ctl.cc.done;
+            __syncwarp();
+            if (all_done) break;
+        }
         // ------------------------------------------------ segment start
 #if LMO_ATTN_PROFILE
         prof_c0 = clock64();

@@ -86,14 +86,15 @@ template <int BN, int MT = 1>
 struct Smem {
     static constexpr int B = BN * 128;                 // BN x 64 fp16, SWIZZLE_128B
     static constexpr int CODES = kM * 32 * MT;         // 4 KB per tile per step
-    static constexpr int META = kM * 4 * kParts * MT;  // per step: one 4-B copy per thread (thread-private)
     static constexpr int OFF_CODES = kX * B;
     static constexpr int PBLK = kM * 32 + kM * 4;      // packed layout: one tile-step = codes | meta (4608 B)
     static constexpr int PSTEP = PBLK * MT;
     static constexpr int CSLOT = PSTEP * kCPS;         // one codes transfer: kCPS steps
-    static constexpr int OFF_META = OFF_CODES + kCodeSlots * CSLOT;
-    static constexpr int OFF_BARS = OFF_META + kCodes * META;
-    static constexpr int BYTES = OFF_BARS + 512 + 1024 /* barriers + TMEM slot; align */;
+    static constexpr int OFF_BARS = OFF_CODES + kCodeSlots * CSLOT;   // (meta: registers / the packed block)
+#ifndef LMO_W4_SMEM_PAD
+#define LMO_W4_SMEM_PAD 0   // (experiments: extra dynamic smem bytes to limit co-resident CTAs)
+#endif
+    static constexpr int BYTES = OFF_BARS + 512 + 1024 /* barriers + TMEM slot; align */ + LMO_W4_SMEM_PAD;
 };
 static_assert((2 * kCodes + 2 * kX + 2 * kStages + 1) * 8 + 4 <= 512, "barrier area");
 template <int BN, int MT = 1>
@@ -101,7 +102,11 @@ struct Tmem {
     static constexpr int ACC = BN * MT;                // accumulator columns (fp32), tile mt at mt * BN
     static constexpr int A0 = BN * MT;                 // A stages: 32 columns per tile (64 fp16 per lane)
     static constexpr int USED = BN * MT + kStages * 32 * MT;
-    static constexpr int COLS = USED <= 32 ? 32 : USED <= 64 ? 64 : USED <= 128 ? 128 : USED <= 256 ? 256 : 512;
+#ifndef LMO_W4_TMEM_COLS
+#define LMO_W4_TMEM_COLS 0   // (experiments: force the TMEM allocation size)
+#endif
+    static constexpr int COLS = LMO_W4_TMEM_COLS ? LMO_W4_TMEM_COLS
+                              : USED <= 32 ? 32 : USED <= 64 ? 64 : USED <= 128 ? 128 : USED <= 256 ? 256 : 512;
     static_assert(USED <= 512, "TMEM");
 };
 
@@ -255,7 +260,6 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
         const int r = tid & (kM - 1), mt = MT == 1 ? 0 : tid >> 7, h = MT == 1 ? tid >> 7 : 0;
         const int tr = mt * kM + r;                              // row within the CTA's rows
         const uint32_t *mrow = meta + (int64_t)(n0 + tr) * (K / kK);
-        const uint32_t meta_u32 = sbase + S::OFF_META + (h * kM * MT + tr) * 4;
         // row-major path: the group meta word of step j is a plain read-only global load issued
         // two steps ahead into registers (L2-resident: 1/16 of the code bytes).
         uint32_t m_next = 0, m_next2 = 0;
@@ -266,7 +270,6 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
             m_next = meta_load(0);
             m_next2 = meta_load(1);
         }
-        (void)meta_u32;
         const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16) + TM::A0 + mt * 32 + h * (WPT / 2);
         // software pipeline: the dequant of step j overlaps the TMEM store of step j-1
         // (tcgen05.wait::st of j-1 only after step j's arithmetic); two register buffers
@@ -295,6 +298,14 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                 m_next2 = meta_load(j + 2);
             }
             const bool last_sub = sub == kCPS - 1 || j == nsteps - 1;
+            // WAR across proxies: the codes (and meta) were read with generic-proxy loads;
+            // the slot is refilled by an async-proxy TMA write once every consumer has
+            // arrived.  The mbarrier release/acquire pair does not order a generic read
+            // before an async-proxy write, and the hardware does issue the arrive while
+            // the shared loads are still in flight: without this fence, rings of 4 or 8
+            // stages corrupted rows nondeterministically (scripts/w4_check.py; DESIGN.md
+            // K7 "root cause").
+            asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
             if (!LMO_W4_WARP_ARRIVE && last_sub) mbar_arrive(&c_empty[cs]);
             const __half2 mn2 = __half2half2(__ushort_as_half((unsigned short)(mw & 0xFFFFu)));
             const __half2 sc2 = __half2half2(__ushort_as_half((unsigned short)(mw >> 16)));
@@ -460,13 +471,13 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
 #endif
 static int w4a16_mt(int N) { return (LMO_W4_MT == 2 && N % (2 * w4::kM) == 0) ? 2 : 1; }
 
-int w4a16_auto_split(int N, int K) {
-    // the most K splits that still fit ONE wave of resident CTAs (2 per SM with one tile per
-    // CTA, 1 with two); measured on the OPT-30B layer GEMMs: more CTAs than one wave (or
-    // a half-empty last wave) costs more than the split-K atomics save
+int w4a16_auto_split(int N, int K, int ctas_per_sm) {
+    // the most K splits that still fit ONE wave of resident CTAs (ctas_per_sm: the occupancy
+    // of the instance being launched); measured on the OPT-30B layer GEMMs: more CTAs than
+    // one wave (or a half-empty last wave) costs more than the split-K atomics save
     const int MT = w4a16_mt(N);
     const int tiles = N / (w4::kM * MT), KB = K / w4::kK;
-    const int slots = device_sm_count() * (MT == 1 ? 2 : 1);
+    const int slots = device_sm_count() * (ctas_per_sm > 0 ? ctas_per_sm : 1);
     int s = slots / tiles;
     if (s > 8) s = 8;
     if (s > KB / 4) s = KB / 4;
@@ -523,8 +534,6 @@ cudaError_t launch_w4a16_pack(const uint8_t *codes, const void *meta, uint8_t *p
 // codes/meta (row-major, 2-D TMA path) or packed (streaming layout, 1-D bulk path)
 cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *packed, const void *x, float *y,
                          int N, int K, int batch, int ksplit, cudaStream_t st) {
-    if (ksplit <= 0) ksplit = w4a16_auto_split(N, K);
-    if (ksplit > K / w4::kK) ksplit = K / w4::kK;
     EncodeTiledFn enc = encode_tiled();
     if (!enc) return cudaErrorNotSupported;
     const int BN = batch <= 64 ? 64 : 128;
@@ -549,15 +558,22 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
             return cudaErrorInvalidValue;
     }
-    if (ksplit > 1) {
-        const cudaError_t e = cudaMemsetAsync(y, 0, (size_t)batch * N * sizeof(float), st);
-        if (e != cudaSuccess) return e;
-    }
     const int MT = w4a16_mt(N);
-    dim3 grid(N / (w4::kM * MT), ksplit);
     const uint32_t *m = static_cast<const uint32_t *>(meta);
+    cudaError_t pre = cudaSuccess;
     auto go = [&](auto kern, int sm, int threads) {
         cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+        if (ksplit <= 0) {   // auto: one wave of the resident CTAs of THIS instance
+            int occ = 0;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, threads, sm);
+            ksplit = w4a16_auto_split(N, K, occ);
+        }
+        if (ksplit > K / w4::kK) ksplit = K / w4::kK;
+        if (ksplit > 1) {
+            pre = cudaMemsetAsync(y, 0, (size_t)batch * N * sizeof(float), st);
+            if (pre != cudaSuccess) return;
+        }
+        dim3 grid(N / (w4::kM * MT), ksplit);
         kern<<<grid, threads, sm, st>>>(tc, tx, m, packed, y, N, K, batch, ksplit);
     };
     constexpr int T1 = w4::Roles<1>::THREADS, T2 = w4::Roles<2>::THREADS;
@@ -576,6 +592,7 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
         if (packed) go(w4::w4a16_kernel<128, true, 1>, w4::Smem<128>::BYTES, T1);
         else go(w4::w4a16_kernel<128, false, 1>, w4::Smem<128>::BYTES, T1);
     }
+    if (pre != cudaSuccess) return pre;
     const cudaError_t e = cudaGetLastError();
     if (e == cudaSuccess) note_launch();
     return e;

@@ -1,0 +1,42 @@
+"""compute-sanitizer over the library: memcheck (out-of-bounds /
+misaligned accesses), racecheck (shared-memory hazards), synccheck (barrier
+misuse) on tests/sanitize_driver.py.  Every tool must report zero errors.
+
+Note: racecheck models generic-proxy shared-memory accesses only; the async-proxy
+(TMA, tcgen05) ordering that broke the W4A16 code ring (K7) is not
+visible to it -- that is covered by test_gpu_w4a16.py's repeat test."""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+DRIVER = os.path.join(ROOT, "tests", "sanitize_driver.py")
+
+
+def sanitizer():
+    for c in (shutil.which("compute-sanitizer"), "/usr/local/cuda/bin/compute-sanitizer"):
+        if c and os.path.exists(c):
+            return c
+    pytest.skip("compute-sanitizer not found")
+
+
+@pytest.mark.parametrize("tool,part", [("memcheck", "all"), ("racecheck", "attn"), ("racecheck", "quant"),
+                                       ("racecheck", "w4a16"), ("synccheck", "all")])
+def test_compute_sanitizer_clean(tool, part):
+    cmd = [sanitizer(), "--tool", tool, "--error-exitcode", "99", "--print-limit", "20"]
+    if tool == "racecheck":
+        cmd += ["--racecheck-report", "all"]      # warnings too (warp-level WAR on the iterators)
+    res = subprocess.run(cmd + [sys.executable, DRIVER, part], capture_output=True, text=True, timeout=900,
+                         cwd=ROOT)
+    out = res.stdout + res.stderr
+    print(out[-3000:])
+    assert res.returncode == 0, out[-3000:]
+    assert "OK" in res.stdout
+    if tool == "racecheck":
+        assert "RACECHECK SUMMARY: 0 hazards displayed (0 errors, 0 warnings)" in out, out[-2000:]
+    else:
+        assert "ERROR SUMMARY: 0 errors" in out, out[-2000:]

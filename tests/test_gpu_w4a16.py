@@ -155,3 +155,20 @@ def test_w4a16_packed_layout(lmo, N, K, batch, k_split):
     wdq = oracle.dequantize_groupwise(codes, meta, N, K, 1).reshape(N, K).astype(np.float64)
     bound = np.abs(x.cpu().numpy().astype(np.float64)) @ np.abs(wdq).T * 2.0 ** -10 + 1e-6
     assert np.all(np.abs(ys - ref) <= bound)
+
+
+def test_w4a16_row_major_ring_repeatable(lmo):
+    """The row-major path's code ring (2-D TMA refills after generic-proxy reads, DESIGN.md
+    K7 root cause): at the OPT-30B FFN1 shape, 8 back-to-back runs are bit-identical to
+    each other and to the packed path (same arithmetic, 1-D bulk copies)."""
+    g = torch.Generator(device="cuda")
+    g.manual_seed(3)
+    N, K, B = 28672, 7168, 64
+    W = (torch.randn(N, K, generator=g, device="cuda") * 0.02).half()
+    c, m = lmo.lmo_quantize_groupwise(W, N, K, 1)
+    x = torch.randn(B, K, generator=g, device="cuda").half()
+    c, m = c.view(N, K // 2), m.view(N, K // 64)
+    ref = lmo.lmo_w4a16_linear_packed(lmo.lmo_w4a16_pack(c, m, N, K), N, K, x, k_split=1)
+    for _ in range(8):
+        y = lmo.lmo_w4a16_linear(c, m, N, K, x, k_split=1)
+        assert torch.equal(y, ref)

@@ -189,8 +189,15 @@ lmo_status lmo_decode_attention_q4(const lmo_kv_cache *cache, const void *q_f16,
  *        those old-token blocks before the previous kernel has finished
  *        (programmatic dependent launch), overlapping its pipeline fill with
  *        the previous kernel's tail.  Ignored with seq_lens_dev.  0 = none.
+ *        LMO_STEP_FLEXGEN_EXACT = the new token enters its OWN step's attention
+ *        with its raw fp16 K/V (FlexGen's semantics, reading 13b:
+ *        "the new KV cache is compressed, old only decompressed", P:159,
+ *        P:235-243); it is still appended quantized at slot L_b - 1 for later
+ *        steps.  Default (0): the new token is attended through its quantized
+ *        form (reading 13).  Flags combine with |.
  * ------------------------------------------------------------------------- */
 #define LMO_STEP_CACHE_STABLE 1u
+#define LMO_STEP_FLEXGEN_EXACT 2u
 lmo_status lmo_decode_step_q4(const lmo_kv_cache *cache, const void *k_new_f16,
                               const void *v_new_f16, const void *q_f16, int32_t q_heads,
                               int32_t len, const int32_t *seq_lens_dev, float softmax_scale,

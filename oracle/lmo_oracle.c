@@ -37,6 +37,11 @@
  *   Q8 byte[j] = code[2j] | code[2j+1] << 4 (low nibble = even element).
  *   D1 y = RN16(RN32(code * scale + mn))  (Eq 11 in step form).
  *   T1-T5 attention in fp64 on the exact dequantized reals mn + c*scale.
+ *   T6 (reading 13b, FlexGen-exact, optional): the newest token L_b-1 of each
+ *      (b, kv head) enters its own step's attention with its raw fp16 K/V
+ *      (k_last/v_last), not its quantized form -- "the newly generated KV cache
+ *      is quantized" for later steps while the current step computes with it
+ *      (P:159).
  * Each RN32 step is emulated by computing in fp64 and casting to float: the
  * fp64 result of +,-,*,/ on fp32/fp16 operands is either exact or a single
  * RN64 rounding, and RN32(RN64(r)) == RN32(r) because 53 >= 2*24+2.
@@ -232,6 +237,7 @@ typedef struct {
     int B, Hkv, cap, d, Hq;
     const uint16_t *q;
     const int32_t *lens;
+    const uint16_t *k_last, *v_last;   /* T6: raw new-token K/V [B][Hkv][d] or NULL */
     double sigma;
     double *out;
     int64_t row_begin, row_end;  /* rows = b*Hq + h */
@@ -260,10 +266,13 @@ static void attn_rows(attn_job *jb) {
         const uint16_t *qr = jb->q + row * d;
         int64_t base = ((int64_t)b * jb->Hkv + kvh) * jb->cap;
         double m = -INFINITY;
+        const uint16_t *kl = jb->k_last ? jb->k_last + ((int64_t)b * jb->Hkv + kvh) * d : NULL;
+        const uint16_t *vl = jb->v_last ? jb->v_last + ((int64_t)b * jb->Hkv + kvh) * d : NULL;
         for (int j = 0; j < L; ++j) {                       /* T3 */
             double acc = 0.0;
             for (int i = 0; i < d; ++i)
-                acc += lmo_oracle_h2d(qr[i]) * deq_elem(jb->k_codes, jb->k_meta, base + j, d, i);
+                acc += lmo_oracle_h2d(qr[i]) * ((kl && j == L - 1) ? lmo_oracle_h2d(kl[i])        /* T6 */
+                                                                  : deq_elem(jb->k_codes, jb->k_meta, base + j, d, i));
             z[j] = jb->sigma * acc;
             if (z[j] > m) m = z[j];
         }
@@ -273,7 +282,8 @@ static void attn_rows(attn_job *jb) {
         for (int i = 0; i < d; ++i) {
             double acc = 0.0;
             for (int j = 0; j < L; ++j)
-                acc += z[j] * deq_elem(jb->v_codes, jb->v_meta, base + j, d, i);
+                acc += z[j] * ((vl && j == L - 1) ? lmo_oracle_h2d(vl[i])                          /* T6 */
+                                                  : deq_elem(jb->v_codes, jb->v_meta, base + j, d, i));
             o[i] = acc / l;
         }
     }
@@ -284,12 +294,15 @@ static void *attn_thread(void *arg) { attn_rows((attn_job *)arg); return NULL; }
 
 /* o[b][h] = softmax(sigma * q[b][h] . K[b][h/G][0:L_b]) @ V[b][h/G][0:L_b],
  * over the exact dequantized q4 cache.  q: [B][Hq][d] fp16 bits, lens: [B],
- * out: [B][Hq][d] doubles.  nthreads >= 1 splits rows across pthreads. */
-int lmo_oracle_decode_attention_q4_mt(const uint8_t *k_codes, const uint16_t *k_meta,
-                                      const uint8_t *v_codes, const uint16_t *v_meta, int B,
-                                      int Hkv, int cap, int d, const uint16_t *q, int Hq,
-                                      const int32_t *lens, double sigma, double *out,
-                                      int nthreads) {
+ * out: [B][Hq][d] doubles.  nthreads >= 1 splits rows across pthreads.
+ * k_last/v_last (T6, FlexGen-exact): NULL, or raw fp16 K/V [B][Hkv][d] used for
+ * token L_b - 1 instead of its cache slot. */
+int lmo_oracle_decode_attention_q4_ext(const uint8_t *k_codes, const uint16_t *k_meta,
+                                       const uint8_t *v_codes, const uint16_t *v_meta, int B,
+                                       int Hkv, int cap, int d, const uint16_t *q, int Hq,
+                                       const int32_t *lens, const uint16_t *k_last,
+                                       const uint16_t *v_last, double sigma, double *out,
+                                       int nthreads) {
     if (d % 64 != 0 || Hkv <= 0 || Hq % Hkv != 0 || nthreads < 1) return LMO_ORACLE_EINVAL;
     int64_t rows = (int64_t)B * Hq;
     if (nthreads > rows) nthreads = (int)(rows > 0 ? rows : 1);
@@ -297,8 +310,8 @@ int lmo_oracle_decode_attention_q4_mt(const uint8_t *k_codes, const uint16_t *k_
     pthread_t *th = (pthread_t *)calloc((size_t)nthreads, sizeof(pthread_t));
     if (!jobs || !th) { free(jobs); free(th); return LMO_ORACLE_EINVAL; }
     for (int t = 0; t < nthreads; ++t) {
-        attn_job j = {k_codes, v_codes, k_meta, v_meta, B, Hkv, cap, d, Hq, q, lens, sigma, out,
-                      rows * t / nthreads, rows * (t + 1) / nthreads, 0};
+        attn_job j = {k_codes, v_codes, k_meta, v_meta, B, Hkv, cap, d, Hq, q, lens, k_last, v_last,
+                      sigma, out, rows * t / nthreads, rows * (t + 1) / nthreads, 0};
         jobs[t] = j;
     }
     for (int t = 1; t < nthreads; ++t) pthread_create(&th[t], NULL, attn_thread, &jobs[t]);
@@ -311,6 +324,15 @@ int lmo_oracle_decode_attention_q4_mt(const uint8_t *k_codes, const uint16_t *k_
     free(jobs);
     free(th);
     return rc;
+}
+
+int lmo_oracle_decode_attention_q4_mt(const uint8_t *k_codes, const uint16_t *k_meta,
+                                      const uint8_t *v_codes, const uint16_t *v_meta, int B,
+                                      int Hkv, int cap, int d, const uint16_t *q, int Hq,
+                                      const int32_t *lens, double sigma, double *out,
+                                      int nthreads) {
+    return lmo_oracle_decode_attention_q4_ext(k_codes, k_meta, v_codes, v_meta, B, Hkv, cap, d, q,
+                                              Hq, lens, NULL, NULL, sigma, out, nthreads);
 }
 
 int lmo_oracle_decode_attention_q4(const uint8_t *k_codes, const uint16_t *k_meta,

@@ -53,8 +53,11 @@ def lib():
         L.lmo_oracle_decode_attention_q4_mt.argtypes = [P, P, P, P, i32, i32, i32, i32, P, i32, P,
                                                         ctypes.c_double, P, i32]
         L.lmo_oracle_w4a16_linear.argtypes = [P, P, i64, i64, i32, P, i64, P]
+        L.lmo_oracle_decode_attention_q4_ext.argtypes = [P, P, P, P, i32, i32, i32, i32, P, i32, P, P, P,
+                                                         ctypes.c_double, P, i32]
         for f in ("lmo_oracle_quantize_groupwise", "lmo_oracle_dequantize_groupwise", "lmo_oracle_w4a16_linear",
-                  "lmo_oracle_kv_append_quant", "lmo_oracle_decode_attention_q4_mt"):
+                  "lmo_oracle_kv_append_quant", "lmo_oracle_decode_attention_q4_mt",
+                  "lmo_oracle_decode_attention_q4_ext"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -146,9 +149,12 @@ def kv_append_quant(cache: dict, k_new: np.ndarray, v_new: np.ndarray, pos) -> N
 
 
 def decode_attention_q4(cache: dict, q: np.ndarray, lens, sigma: float | None = None,
-                        nthreads: int = 1) -> np.ndarray:
+                        nthreads: int = 1, k_last: np.ndarray | None = None,
+                        v_last: np.ndarray | None = None) -> np.ndarray:
     """softmax(sigma * q K^T) V over the exact dequantized q4 cache,
-    kv head = h // (Hq/Hkv).  q: fp16 [B][Hq][d]; returns float64 [B][Hq][d]."""
+    kv head = h // (Hq/Hkv).  q: fp16 [B][Hq][d]; returns float64 [B][Hq][d].
+    k_last/v_last (reading 13b, FlexGen-exact, T6): raw fp16 [B][Hkv][d] K/V used for
+    token L_b-1 of every (b, kv head) instead of its quantized cache slot."""
     B, Hkv, cap, half = cache["k_codes"].shape
     d = half * 2
     Hq = q.shape[1]
@@ -158,9 +164,14 @@ def decode_attention_q4(cache: dict, q: np.ndarray, lens, sigma: float | None = 
     lens = np.ascontiguousarray(np.broadcast_to(np.asarray(lens, dtype=np.int32), (B,)))
     qb = _bits(q)
     out = np.zeros((B, Hq, d), dtype=np.float64)
-    rc = lib().lmo_oracle_decode_attention_q4_mt(
+    kl = vl = None
+    if k_last is not None or v_last is not None:
+        kl = _bits(np.asarray(k_last, dtype=np.float16).reshape(B, Hkv, d))
+        vl = _bits(np.asarray(v_last, dtype=np.float16).reshape(B, Hkv, d))
+    rc = lib().lmo_oracle_decode_attention_q4_ext(
         _ptr(cache["k_codes"]), _ptr(cache["k_meta"]), _ptr(cache["v_codes"]),
-        _ptr(cache["v_meta"]), B, Hkv, cap, d, _ptr(qb), Hq, _ptr(lens), float(sigma), _ptr(out),
+        _ptr(cache["v_meta"]), B, Hkv, cap, d, _ptr(qb), Hq, _ptr(lens),
+        None if kl is None else _ptr(kl), None if vl is None else _ptr(vl), float(sigma), _ptr(out),
         int(nthreads))
     if rc:
         raise ValueError("oracle attention: invalid arguments")

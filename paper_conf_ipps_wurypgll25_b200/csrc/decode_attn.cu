@@ -181,6 +181,9 @@ struct AttnArgs {
     const __half *k_new;      // fused append (team mode): [B][Hkv][D] new token K, or nullptr
     const __half *v_new;      //                            new token V
     int early;                // prefetch the old-token cache before griddepcontrol.wait
+    int flex;                 // LMO_STEP_FLEXGEN_EXACT: slot L-1 is attended with the raw fp16
+    const __half *raw_k;      //   k_new / v_new [B][Hkv][D] instead of its quantized form
+    const __half *raw_v;
     int prof_slot;            // (LMO_ATTN_PROFILE builds) record slot of this launch
     WorkMap wm;               // host-computed work map (uniform length; completed on device
                               // from the length prefix in per-sequence mode)
@@ -858,7 +861,9 @@ decode_attn_q4_kernel(const AttnArgs a) {
             cc.template next<SCH>(wms);
         }
         __syncwarp();
-        const int seg_n = ctl.seg.sn, blk0 = ctl.seg.blk0, L = ctl.seg.L;
+        // L: tokens taken from the q4 cache (FlexGen-exact: all but the new token at L-1,
+        // which the pair's last segment adds from its raw fp16 K/V in the epilogue)
+        const int seg_n = ctl.seg.sn, blk0 = ctl.seg.blk0, L = ctl.seg.L - a.flex;
         const int Lseg = min(L, (blk0 + seg_n) * kBlk);   // end (exclusive) of this segment's tokens
 #if LMO_ATTN_PROFILE
         ++prof_seg;
@@ -905,7 +910,10 @@ decode_attn_q4_kernel(const AttnArgs a) {
         // sets it; afterwards it only decreases (a stage whose scale * 2^Ei >= 2^15).
         int Ei = 0;
         uint32_t vthr = 0x10000u;                 // V meta word >= vthr <=> scale >= 2^(15 - Ei)
-        float mE[2] = {NEG_INF, NEG_INF};
+        // (finite sentinel while no token has been seen: a segment whose tokens are all
+        // masked -- FlexGen-exact's last block -- then gets p = exp2(-inf - sentinel) = 0
+        // instead of exp2(-inf + inf) = NaN; records store -inf for it, see rec_m)
+        float mE[2] = {-1e30f, -1e30f};
         // rare, warp-uniform: lower Ei to fit the largest V scale vx (meta word) of the warp;
         // returns the factor applied to l, Pm and acc (the caller rescales its live p)
         auto v_exp = [&](uint32_t vx) -> float {
@@ -1344,6 +1352,53 @@ decode_attn_q4_kernel(const AttnArgs a) {
                 }
         const SegDesc sd = ctl.seg;
         const int64_t rowbase = (int64_t)sd.b * a.Hq + (int64_t)sd.kvh * a.G;
+        if (a.flex && sd.L > 0 && sd.blk0 + sd.sn == sd.nb) {
+            // FlexGen-exact (NEXT-1; reading 13b): the new token's own K/V enter its
+            // attention unquantized.  Lane (g, t) owns dims grp*64 + 8g .. +7 of heads 2t, 2t+1
+            // (MHA: head 0): z_new = sigma*log2e * q.k_new (fp32, reduced over g), merged into
+            // the running softmax with the same 2^Ei factor as l, Pm and acc.
+            const int64_t pr = ((int64_t)sd.b * a.Hkv + sd.kvh) * D;
+            float z[2];
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+                const int h = MHA ? 0 : min(2 * t + e, a.G - 1);
+                const __half *qp = a.q + (rowbase + h) * D;
+                float dot = 0.f;
+#pragma unroll
+                for (int grp = 0; grp < NG; ++grp) {
+                    const uint4 qw = *reinterpret_cast<const uint4 *>(qp + grp * 64 + 8 * g);
+                    const uint4 kw = *reinterpret_cast<const uint4 *>(a.raw_k + pr + grp * 64 + 8 * g);
+                    const __half2 *qh = reinterpret_cast<const __half2 *>(&qw);
+                    const __half2 *kh = reinterpret_cast<const __half2 *>(&kw);
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const float2 qf2 = __half22float2(qh[i]), kf2 = __half22float2(kh[i]);
+                        dot = fmaf(qf2.x, kf2.x, fmaf(qf2.y, kf2.y, dot));
+                    }
+                }
+                z[e] = sum_over_g(dot) * zs;
+            }
+#pragma unroll
+            for (int e = 0; e < 2; ++e) {
+                const float m2 = fmaxf(m_run[e], z[e]);
+                const float sc = fast_exp2(mE[e] - (m2 - (float)Ei));     // old terms (0 if none)
+                const float pn = fast_exp2(z[e] - m2) * exp2i(Ei);
+                lt[e] = fmaf(lt[e], sc, pn);
+#pragma unroll
+                for (int grp = 0; grp < NG; ++grp) {
+                    const uint4 vw = *reinterpret_cast<const uint4 *>(a.raw_v + pr + grp * 64 + 8 * g);
+                    const __half2 *vh = reinterpret_cast<const __half2 *>(&vw);
+#pragma unroll
+                    for (int i = 0; i < 4; ++i) {
+                        const float2 v2 = __half22float2(vh[i]);
+                        vo[e][grp][2 * i] = fmaf(vo[e][grp][2 * i], sc, pn * v2.x);
+                        vo[e][grp][2 * i + 1] = fmaf(vo[e][grp][2 * i + 1], sc, pn * v2.y);
+                    }
+                }
+                m_run[e] = m2;
+                mE[e] = m2 - (float)Ei;
+            }
+        }
         const bool full = SCH == 1 || (SCH == 0 && (sd.blk0 == 0) && (sd.sn == sd.nb) && wms.T <= 1);
         if (SCH == 2 || (SCH == 0 && wms.T > 1)) {
             // ---- pair team: partials through L2 scratch, named barrier, rank 0 merges
@@ -1361,7 +1416,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
                         __stcg(r4 + 1, make_float4(vo[e][grp][4], vo[e][grp][5], vo[e][grp][6], vo[e][grp][7]));
                     }
                     if (g == 0) {
-                        __stcg(rec + h * GG::REC + D, mE[e]);
+                        __stcg(rec + h * GG::REC + D, m_run[e] == NEG_INF ? NEG_INF : mE[e]);
                         __stcg(rec + h * GG::REC + D + 1, lt[e]);
                     }
                 }
@@ -1454,7 +1509,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
                         __stcg(r4 + 1, make_float4(vo[e][grp][4], vo[e][grp][5], vo[e][grp][6], vo[e][grp][7]));
                     }
                     if (g == 0) {
-                        __stcg(rec + h * GG::REC + D, mE[e]);
+                        __stcg(rec + h * GG::REC + D, m_run[e] == NEG_INF ? NEG_INF : mE[e]);
                         __stcg(rec + h * GG::REC + D + 1, lt[e]);
                     }
                 }
@@ -1756,6 +1811,9 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
                                     const void *k_new, const void *v_new, unsigned flags) {
     AttnArgs a;
     a.early = (flags & LMO_STEP_CACHE_STABLE) ? 1 : 0;
+    a.flex = (k_new && (flags & LMO_STEP_FLEXGEN_EXACT)) ? 1 : 0;
+    a.raw_k = static_cast<const __half *>(k_new);
+    a.raw_v = static_cast<const __half *>(v_new);
     a.k_new = static_cast<const __half *>(k_new);
     a.v_new = static_cast<const __half *>(v_new);
     a.kv = c.kv;

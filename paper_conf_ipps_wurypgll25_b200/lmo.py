@@ -20,6 +20,7 @@ LMO_OK, LMO_ERR_NULL, LMO_ERR_SHAPE, LMO_ERR_UNSUPPORTED, LMO_ERR_ALIGN, LMO_ERR
     LMO_ERR_CUDA = range(7)
 LMO_F16, LMO_F32 = 0, 1
 LMO_STEP_CACHE_STABLE = 1
+LMO_STEP_FLEXGEN_EXACT = 2  # the new token attends with its raw fp16 K/V (include/lmo.h)
 LMO_SPLITS_STREAMK = -1   # num_splits value selecting the stream-K schedule
 LMO_SPLITS_SMTEAM = -2    # num_splits value selecting the SM-team schedule
 GROUP = 64

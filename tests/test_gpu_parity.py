@@ -620,3 +620,75 @@ def test_sharded_step_bit_identical(lmo, G, d):
     hi, kv_hi = run(B // 2, B // 2)
     assert torch.equal(torch.cat([lo, hi]), full)
     assert torch.equal(torch.cat([kv_lo, kv_hi]), kv_full)
+
+
+# ------------------------------------ NEXT-1: FlexGen-exact step (reading 13b) --
+
+@pytest.mark.parametrize("B,Hkv,G,d,L,ns,flags", [
+    (4, 6, 1, 128, 300, 0, 0), (2, 2, 8, 128, 129, 0, 0), (3, 4, 2, 64, 77, 2, 0), (2, 3, 1, 128, 40, 4, 0),
+    (2, 2, 4, 128, 200, 3, 0), (1, 2, 1, 128, 1, 0, 0), (2, 2, 8, 128, 1, 0, 0), (3, 5, 1, 128, 33, -1, 0),
+    (3, 4, 8, 128, 129, -1, 0), (4, 6, 1, 128, 300, -2, 0), (2, 2, 8, 128, 16, 0, 0), (2, 2, 8, 128, 17, 0, 0),
+    (4, 6, 1, 128, 300, 0, 1), (2, 2, 8, 128, 129, 0, 1), (64, 9, 1, 128, 47, 0, 1)])
+def test_decode_step_flexgen_exact(lmo, B, Hkv, G, d, L, ns, flags):
+    """LMO_STEP_FLEXGEN_EXACT: the new token's raw fp16 K/V in its own attention (oracle T6),
+    while the cache still receives its quantized row at slot L-1 (bit-exact)."""
+    seed = 77 + L + G
+    cap = L + 7
+    kf = torch.empty((B, Hkv, L, d), dtype=torch.float16, device="cuda")
+    vf = torch.empty_like(kf)
+    lmo.lmo_gen_fill_f16(kf, seed, I.STREAM_K, 0, 0, 0, 0)
+    lmo.lmo_gen_fill_f16(vf, seed, I.STREAM_V, 0, 0, 0, 0)
+    cache = lmo.KVCache.empty(B, Hkv, cap, d)
+    cache.kv.fill_(0x3C)
+    if L > 1:
+        lmo.lmo_kv_append_quant(cache, kf[:, :, :L - 1].contiguous(), vf[:, :, :L - 1].contiguous(), 0)
+    q = torch.empty((B, Hkv * G, 1, d), dtype=torch.float16, device="cuda")
+    lmo.lmo_gen_fill_f16(q, seed, I.STREAM_Q, 0, 0, 0, 0, group=G)
+    q = q.view(B, Hkv * G, d)
+    kn, vn = kf[:, :, L - 1].contiguous(), vf[:, :, L - 1].contiguous()
+    out = lmo.lmo_decode_step_q4(cache, kn, vn, q, L, num_splits=ns,
+                                 flags=lmo.LMO_STEP_FLEXGEN_EXACT | (lmo.LMO_STEP_CACHE_STABLE if flags else 0))
+    torch.cuda.synchronize()
+    host = oracle.new_cache(B, Hkv, cache.capacity, d)
+    oracle.kv_append_quant(host, kf.cpu().numpy(), vf.cpu().numpy(), 0)
+    got = cache_to_host(cache)
+    for key in host:
+        assert np.array_equal(got[key][:, :, :L], host[key][:, :, :L]), key
+    ref = oracle.decode_attention_q4(host, q.cpu().numpy(), L, nthreads=8, k_last=kn.cpu().numpy(),
+                                     v_last=vn.cpu().numpy())
+    o = out.cpu().numpy()
+    check_attention(o, ref, f"flexgen B{B} Hkv{Hkv} G{G} d{d} L{L} ns{ns} flags{flags}")
+    if L == 1:   # closed form: the raw V row (fp32 of fp16) within rounding of the 1/l normalisation
+        want = np.repeat(vn.cpu().numpy().astype(np.float64), G, axis=1)
+        assert np.max(np.abs(o - want)) <= 1e-6 * max(1.0, np.abs(want).max())
+
+
+def test_decode_step_flexgen_exact_per_sequence_lengths(lmo):
+    B, Hkv, G, d, cap = 5, 3, 2, 128, 208
+    lens = np.array([200, 1, 0, 65, 129], np.int32)
+    kf = torch.empty((B, Hkv, cap, d), dtype=torch.float16, device="cuda")
+    vf = torch.empty_like(kf)
+    lmo.lmo_gen_fill_f16(kf, 19, I.STREAM_K, 0, 0, 0, 0)
+    lmo.lmo_gen_fill_f16(vf, 19, I.STREAM_V, 0, 0, 0, 0)
+    cache = lmo.KVCache.empty(B, Hkv, cap, d)
+    lmo.lmo_kv_append_quant(cache, kf, vf, 0)
+    kn = (torch.randn((B, Hkv, d), device="cuda") * 2).half()
+    vn = torch.randn((B, Hkv, d), device="cuda").half()
+    q = torch.empty((B, Hkv * G, 1, d), dtype=torch.float16, device="cuda")
+    lmo.lmo_gen_fill_f16(q, 19, I.STREAM_Q, 0, 0, 0, 0, group=G)
+    q = q.view(B, Hkv * G, d)
+    out = lmo.lmo_decode_step_q4(cache, kn, vn, q, 0, seq_lens=dev(lens), flags=lmo.LMO_STEP_FLEXGEN_EXACT)
+    torch.cuda.synchronize()
+    kh, vh = kf.cpu().numpy().copy(), vf.cpu().numpy().copy()
+    for b in range(B):
+        if lens[b] > 0:
+            kh[b, :, lens[b] - 1] = kn.cpu().numpy()[b]
+            vh[b, :, lens[b] - 1] = vn.cpu().numpy()[b]
+    host = oracle.new_cache(B, Hkv, cache.capacity, d)
+    oracle.kv_append_quant(host, kh, vh, 0)
+    ref = oracle.decode_attention_q4(host, q.cpu().numpy(), np.maximum(lens, 1), nthreads=8,
+                                     k_last=kn.cpu().numpy(), v_last=vn.cpu().numpy())
+    o = out.cpu().numpy()
+    keep = lens > 0
+    assert np.all(o[~keep] == 0)
+    check_attention(o[keep], ref[keep], "flexgen per-sequence lengths")

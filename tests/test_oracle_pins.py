@@ -361,6 +361,71 @@ def test_attention_brute_force_tiny(L, d, Hq, Hkv):
             assert np.max(np.abs(out[b, h] - ref)) <= 1e-12 * max(1.0, np.max(np.abs(ref)))
 
 
+# ------------------------------- T6: FlexGen-exact new token (reading 13b) --
+
+def test_flexgen_exact_single_token_is_raw_v():
+    """Closed form: with L = 1 the only token has softmax weight 1, so the output is
+    the new token's RAW fp16 V row exactly (not its 4-bit reconstruction)."""
+    rng = np.random.default_rng(RNG_SEED + 30)
+    d, B, Hkv, G = 128, 2, 3, 2
+    cache = random_cache(rng, B, Hkv, 4, d)
+    k_last = (rng.standard_normal((B, Hkv, d)) * 3).astype(np.float16)
+    v_last = (rng.standard_normal((B, Hkv, d)) * 0.7).astype(np.float16)
+    q = rng.standard_normal((B, Hkv * G, d)).astype(np.float16)
+    o = oracle.decode_attention_q4(cache, q, 1, k_last=k_last, v_last=v_last)
+    for b in range(B):
+        for h in range(Hkv * G):
+            assert np.array_equal(o[b, h], v_last[b, h // G].astype(np.float64))
+    # and the quantized path does NOT reproduce it (v_last is off the q4 grid)
+    oq = oracle.decode_attention_q4(cache, q, 1)
+    assert not np.array_equal(oq, o)
+
+
+@pytest.mark.parametrize("L,d,Hq,Hkv", [(2, 64, 2, 2), (6, 64, 4, 2), (5, 128, 2, 1)])
+def test_flexgen_exact_brute_force_tiny(L, d, Hq, Hkv):
+    """Independent brute force: tokens 0..L-2 from the exact dequantized cache, token L-1
+    from the raw fp16 K/V (math.fsum, no max subtraction)."""
+    rng = np.random.default_rng(RNG_SEED + 31 + L)
+    B = 2
+    cache = random_cache(rng, B, Hkv, L, d)
+    k_last = (rng.standard_normal((B, Hkv, d)) * 1.5).astype(np.float16)
+    v_last = rng.standard_normal((B, Hkv, d)).astype(np.float16)
+    q = rng.standard_normal((B, Hq, d)).astype(np.float16)
+    sigma = 1 / math.sqrt(d)
+    out = oracle.decode_attention_q4(cache, q, L, sigma, k_last=k_last, v_last=v_last)
+    G = Hq // Hkv
+    for b in range(B):
+        for h in range(Hq):
+            kv = h // G
+            kr = exact_rows(cache, "k", b, kv, L - 1) + [[Fraction(float(x)) for x in k_last[b, kv]]]
+            vr = exact_rows(cache, "v", b, kv, L - 1) + [[Fraction(float(x)) for x in v_last[b, kv]]]
+            ref = brute_attention(q[b, h], kr, vr, sigma)
+            assert np.max(np.abs(out[b, h] - ref)) <= 1e-12 * max(1.0, np.max(np.abs(ref)))
+
+
+def test_flexgen_exact_equals_quantized_on_grid():
+    """When the new token's K/V lie on their own q4 grid (mn + k*step with a power-of-two
+    step, codes 0..15 present), quantization loses nothing, so the FlexGen-exact and the
+    quantized readings coincide exactly."""
+    rng = np.random.default_rng(RNG_SEED + 32)
+    B, Hkv, d, L = 2, 2, 128, 9
+    k = (rng.standard_normal((B, Hkv, L, d))).astype(np.float16)
+    v = (rng.standard_normal((B, Hkv, L, d))).astype(np.float16)
+    for x in (k, v):                                  # last token on-grid, every group
+        for b in range(B):
+            for h in range(Hkv):
+                for gi in range(d // 64):
+                    kk = rng.integers(0, 16, 64)
+                    kk[:2] = [0, 15]
+                    x[b, h, L - 1, gi * 64:(gi + 1) * 64] = (-1.0 + kk * 0.125).astype(np.float16)
+    cache = oracle.new_cache(B, Hkv, L, d)
+    oracle.kv_append_quant(cache, k, v, 0)
+    q = rng.standard_normal((B, Hkv, d)).astype(np.float16)
+    a = oracle.decode_attention_q4(cache, q, L)
+    f = oracle.decode_attention_q4(cache, q, L, k_last=k[:, :, L - 1], v_last=v[:, :, L - 1])
+    assert np.array_equal(a, f)
+
+
 def test_attention_closed_forms():
     rng = np.random.default_rng(RNG_SEED + 9)
     d, L = 64, 6

@@ -1,0 +1,66 @@
+"""NEXT-4: the paper's performance model (Eq 1-24) re-parameterised for B200
+(costmodel.py) predicts the measured resident and host-offloaded decode steps.
+
+The model's parameters are rates measured independently of these steps (copy
+bandwidth, pinned-copy PCIe bandwidth, the per-SMSP stage cost probe); the
+targets are committed bench lines (tests/golden/measured_b200.json).  Bar: 15%."""
+import json
+import os
+
+import pytest
+
+from paper_conf_ipps_wurypgll25_b200 import configs as C
+from paper_conf_ipps_wurypgll25_b200 import costmodel as M
+
+GOLD = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "measured_b200.json")))
+TIMED_T = [1 + (j * 30) // 19 for j in range(20)]          # bench.py's 20 timed steps over t = 1..31
+
+
+def rel(a, b):
+    return abs(a - b) / b
+
+
+def test_resident_step_c2_within_15pct():
+    w = C.CONFIGS["c2"]
+    pred = sum(M.decode_step_s(w, t) for t in TIMED_T) / len(TIMED_T) * 1e3
+    assert rel(pred, GOLD["c2_resident_ms_per_step"]["value"]) <= 0.15, pred
+
+
+def test_offload_step_c2_within_15pct():
+    """Eq 2 with Eq 6-7: the offloaded step is load_cache-bound (PCIe), compute hidden."""
+    w = C.CONFIGS["c2"]
+    g = GOLD["c2_offload_ms_per_step"]
+    pred = M.decode_step_s(w, g["L"] - w.prompt, offload_kv=True) * 1e3
+    assert rel(pred, g["value"]) <= 0.15, pred
+    st = M.decode_layer(M.Model.from_workload(w), g["L"], M.Hardware(), offload_kv=True)
+    assert st.t_gen() == st.load_cache and st.load_cache > 50 * st.compute
+
+
+@pytest.mark.parametrize("key,gold", [("c4", "c4_attention_us_per_launch"), ("c5", "c5_attention_us_per_launch")])
+def test_attention_kernel_within_15pct(key, gold):
+    w = C.CONFIGS[key]
+    g = GOLD[gold]
+    pred = M.attention_kernel_s(M.Model.from_workload(w), g["L"], M.Hardware()) * 1e6
+    assert rel(pred, g["value"]) <= 0.15, pred
+
+
+def test_paper_reading_and_sizes():
+    """Eq 17-19 sizes at the paper's OPT-30B workload (h1 = 7168, bls = 640, s = 64, n = 128)
+    reproduce the 0.8 GB new-KV-per-token figure (with fp16 and 48 layers), and
+    the paper's unfused reading costs more than the fused one (separate dequant passes)."""
+    m = M.Model(h1=7168, h2=4 * 7168, s=64, n=128, bls=640, l=48, kv_heads=56)
+    assert abs(M.new_kv_cache(m) * 2 * m.l / 2 ** 30 - 0.82) < 0.01
+    assert M.old_kv_cache(m) == 2 * (64 + 64) * 7168 * 640
+    w = C.CONFIGS["c2"]
+    fused = M.decode_step_s(w, 16)
+    paper = M.decode_step_s(w, 16, reading="paper")
+    assert paper > fused
+    # KV quantization pays off when the cache is offloaded (use case 2)
+    r = M.kv_quantization_beneficial(w, 16)
+    assert r["beneficial"] and r["speedup"] > 3.0
+
+
+def test_total_time_eq1_is_sum_of_steps():
+    w = C.CONFIGS["c1"]
+    tot = M.total_time_s(w, t_pf_layer=0.0)
+    assert abs(tot - sum(M.decode_step_s(w, t) for t in range(1, w.gen))) < 1e-12

@@ -319,8 +319,21 @@ __device__ __forceinline__ int tperm(int r) { return r ^ ((r >> 1) & 1); }  // 0
 //   u[2] = (nib2, nib6) * 2^-24, u[3] = (nib3, nib7) * 2^-20.
 // The 2^-20 slots meet q/16 in the MMA (see the q fragments), so every
 // product is q_i c_i 2^-24.
+// x >> 8.  LMO_SHR_FMA: as the high word of x * 2^24 (IMAD.HI on the FMA pipe) -- the
+// unpacking is ALU-pipe bound (LOP3/PRMT/SHF), the FMA pipe is nearly idle.
+#ifndef LMO_SHR_FMA
+#define LMO_SHR_FMA 0
+#endif
+__device__ __forceinline__ uint32_t shr8(uint32_t x) {
+#if LMO_SHR_FMA
+    return __umulhi(x, 1u << 24);
+#else
+    return x >> 8;
+#endif
+}
+
 __device__ __forceinline__ void unpack_k(uint32_t w, uint32_t *u) {
-    const uint32_t s = w >> 8;
+    const uint32_t s = shr8(w);
     u[0] = w & 0x000F000Fu;
     u[1] = w & 0x00F000F0u;
     u[2] = s & 0x000F000Fu;
@@ -332,7 +345,7 @@ __device__ __forceinline__ void unpack_k(uint32_t w, uint32_t *u) {
 __device__ __forceinline__ void unpack_v(uint32_t wa, uint32_t wb, uint32_t *j) {
     const uint32_t lo = prmt(wa, wb, 0x5410u);   // [A.b0, A.b1, B.b0, B.b1]
     const uint32_t hi = prmt(wa, wb, 0x7632u);   // [A.b2, A.b3, B.b2, B.b3]
-    const uint32_t lo8 = lo >> 8, hi8 = hi >> 8;
+    const uint32_t lo8 = shr8(lo), hi8 = shr8(hi);
     j[0] = lo & 0x000F000Fu;
     j[1] = lo & 0x00F000F0u;
     j[2] = lo8 & 0x000F000Fu;
@@ -384,6 +397,18 @@ __device__ __forceinline__ uint32_t movmatrix_t(uint32_t x) {
     uint32_t y;
     asm("movmatrix.sync.aligned.m8n8.trans.b16 %0, %1;\n" : "=r"(y) : "r"(x));
     return y;
+}
+
+#ifndef LMO_REDUX_MAX
+#define LMO_REDUX_MAX 0
+#endif
+// warp-wide float max through redux.sync.max.u32 on an order-preserving integer image
+// (x >= 0: sign bit set; x < 0: all bits flipped); exact, -inf stays -inf
+__device__ __forceinline__ float warp_max_f32(float x) {
+    uint32_t u = __float_as_uint(x);
+    u = (u & 0x80000000u) ? ~u : (u | 0x80000000u);
+    u = __reduce_max_sync(0xffffffffu, u);
+    return __uint_as_float((u & 0x80000000u) ? (u & 0x7FFFFFFFu) : ~u);
 }
 
 __device__ __forceinline__ float max_over_g(float v) {   // lanes with equal t (xor 4, 8, 16)
@@ -1070,9 +1095,13 @@ decode_attn_q4_kernel(const AttnArgs a) {
                 // the running max moves only if some lane's score exceeds it: one vote
                 // instead of a 5-shuffle max chain on most stages (same result)
                 if (!LMO_LAZY_MAX || __any_sync(0xffffffffu, z > m_run[0])) {
+#if LMO_REDUX_MAX
+                const float mb = warp_max_f32(z);              // one REDUX instead of a 5-step shuffle chain
+#else
                 float mb = z;
 #pragma unroll
                 for (int off = 16; off > 0; off >>= 1) mb = fmaxf(mb, __shfl_xor_sync(0xffffffffu, mb, off));
+#endif
                 if (mb > m_run[0]) {                          // warp-uniform
                     const float a0 = fast_exp2(m_run[0] - mb);
                     m_run[0] = mb;

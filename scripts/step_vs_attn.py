@@ -1,0 +1,61 @@
+"""Where does the fused step lose time vs attention alone?  Graph-captured layer
+loops (footprint > L2) of: attention only; fused step (CACHE_STABLE / no flags);
+separate append kernel + attention.  usage: step_vs_attn.py c4 [c2 ...]"""
+import sys, os
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+from paper_conf_ipps_wurypgll25_b200 import lmo
+from paper_conf_ipps_wurypgll25_b200.configs import CONFIGS
+
+for key in sys.argv[1:] or ["c4"]:
+    w = CONFIGS[key]
+    L = w.prompt + w.gen // 2
+    nl = max(4, min(64, int(6.0e9 // (w.batch * w.kv_heads * w.capacity * 144))))
+    caches = []
+    for l in range(nl):
+        c = lmo.KVCache.empty(w.batch, w.kv_heads, w.capacity, w.head_dim)
+        c.kv.random_(0, 256)
+        for nm in ("k_meta", "v_meta"):
+            c.field(nm).view(torch.int32).fill_(0x2C00BC00)
+        caches.append(c)
+    q = torch.randn(w.batch, w.q_heads, w.head_dim, device='cuda').half()
+    kn = torch.randn(w.batch, w.kv_heads, 1, w.head_dim, device='cuda').half()
+    vn = torch.randn_like(kn)
+    out = torch.empty(w.batch, w.q_heads, w.head_dim, device='cuda')
+    ws = lmo.attention_workspace(w.batch, w.kv_heads, w.q_heads, w.head_dim)
+    abis = [c.abi() for c in caches]
+    st = torch.cuda.Stream()
+    variants = {
+        "attn": lambda l: lmo.lmo_decode_attention_q4(caches[l], q, L, out=out, workspace=ws, abi=abis[l], stream=st),
+        "step_stable": lambda l: lmo.lmo_decode_step_q4(caches[l], kn, vn, q, L, out=out, workspace=ws, abi=abis[l],
+                                                        flags=lmo.LMO_STEP_CACHE_STABLE, stream=st),
+        "step_plain": lambda l: lmo.lmo_decode_step_q4(caches[l], kn, vn, q, L, out=out, workspace=ws, abi=abis[l],
+                                                       stream=st),
+        "append+attn": lambda l: (lmo.lmo_kv_append_quant(caches[l], kn, vn, L - 1, abi=abis[l], stream=st),
+                                  lmo.lmo_decode_attention_q4(caches[l], q, L, out=out, workspace=ws, abi=abis[l],
+                                                              stream=st)),
+        "append": lambda l: lmo.lmo_kv_append_quant(caches[l], kn, vn, L - 1, abi=abis[l], stream=st),
+    }
+    res = {}
+    for name, fn in variants.items():
+        with torch.cuda.stream(st):
+            for l in range(nl):
+                fn(l)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=st):
+            for l in range(nl):
+                fn(l)
+        for _ in range(2):
+            g.replay()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        reps = 5
+        with torch.cuda.stream(st):
+            e0.record(st)
+            for _ in range(reps):
+                g.replay()
+            e1.record(st)
+        torch.cuda.synchronize()
+        res[name] = e0.elapsed_time(e1) * 1e3 / (reps * nl)
+    print(key, f"L={L} layers={nl}", "  ".join(f"{k} {v:.1f}us" for k, v in res.items()), flush=True)

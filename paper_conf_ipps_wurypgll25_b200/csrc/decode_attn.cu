@@ -63,6 +63,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_GQA_VOTE
 #define LMO_GQA_VOTE 1   // GQA FULL stages: rescale only when a running max moved (one vote)
 #endif
+#ifndef LMO_EARLY_TEST
+#define LMO_EARLY_TEST 0   // non-blocking mbarrier test of stage i+2 during iteration i
+#endif
 #ifndef LMO_NO_SCH
 #define LMO_NO_SCH 0     // 1: every schedule runs the generic kernel instance (experiments)
 #endif
@@ -765,14 +768,17 @@ decode_attn_q4_kernel(const AttnArgs a) {
     auto app_src = [&](int p) {
         return (kvsel == 0 ? a.k_new : a.v_new) + (int64_t)p * D + grp8 * 64 + lane8 * 8;
     };
-    uint4 xv_first = make_uint4(0, 0, 0, 0);
+    uint4 xv_first = make_uint4(0, 0, 0, 0), xv_second = make_uint4(0, 0, 0, 0);
     uint4 qraw[NG][2];
     // Team mode knows the warp's first pair: issue its q and new-token loads, then
     // (non-early) the bulk copies, and only then consume the loads -- the small loads
     // are queued ahead of the stage traffic and their latencies overlap.
     auto fetch_first = [&]() {
-        if (app_warp && lane_ok && app_lo < app_hi)
+        if (app_warp && lane_ok && app_lo < app_hi) {
             xv_first = *reinterpret_cast<const uint4 *>(app_src(app_lo));
+            if (app_lo + app_step < app_hi)      // the warp's second pair: load now, overlapped
+                xv_second = *reinterpret_cast<const uint4 *>(app_src(app_lo + app_step));
+        }
         if (TEAMK || wms.T) {
             fb = (int)wms.dHkv.div((uint32_t)p_first);
             fk = p_first - fb * a.Hkv;
@@ -796,8 +802,8 @@ decode_attn_q4_kernel(const AttnArgs a) {
             for (int p = app_lo; p < app_hi; p += app_step) {
                 const int b = (int)wms.dHkv.div((uint32_t)p);
                 const int Lb = a.lens ? min(a.lens[b], a.cap) : a.len;
-                uint4 xv = xv_first;
-                if (p != app_lo && lane_ok) xv = *reinterpret_cast<const uint4 *>(app_src(p));
+                uint4 xv = p == app_lo ? xv_first : xv_second;
+                if (p > app_lo + app_step && lane_ok) xv = *reinterpret_cast<const uint4 *>(app_src(p));
                 uint32_t mw;
                 const uint32_t w = quantize_group_lane8(xv, mw);
                 if (lane_ok && Lb >= 1) {
@@ -818,6 +824,28 @@ decode_attn_q4_kernel(const AttnArgs a) {
     // (Stream-K / SM teams learn their first pair from the producer prologue.)
     prologue_setup();
     if (early) {
+        // L2 prefetch, ahead of the stage copies, of what the wait releases: the first pair's
+        // q rows and the new-token K/V rows of the warp's first two appending pairs.  A
+        // prefetch only warms L2 (the point of coherence; L1 is not filled): the loads after
+        // the wait still see the producer's writes.
+        if (TEAMK || wms.T) {
+            const int p0 = p_first;
+            if (p0 < a.B * a.Hkv) {
+                const int b0 = (int)wms.dHkv.div((uint32_t)p0), k0 = p0 - b0 * a.Hkv;
+                const char *qb = reinterpret_cast<const char *>(a.q + ((int64_t)b0 * a.Hq + (int64_t)k0 * a.G) * D);
+                const int qlines = a.G * D * 2 / 128;
+                if (lane < qlines) asm volatile("prefetch.global.L2 [%0];" ::"l"(qb + lane * 128));
+            }
+            if (app_warp && lane < 4 * NG) {
+                const int pa = app_lo + (lane >= 2 * NG ? app_step : 0);
+                if (pa < app_hi) {
+                    const int part = lane % (2 * NG);            // K lines then V lines of one row
+                    const __half *src = (part < NG ? a.k_new : a.v_new) + (int64_t)pa * D;
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(reinterpret_cast<const char *>(src) +
+                                                                    (part % NG) * 128));
+                }
+            }
+        }
         prologue(true);
         asm volatile("griddepcontrol.wait;\n" ::: "memory");
         fetch_first();
@@ -1286,13 +1314,20 @@ decode_attn_q4_kernel(const AttnArgs a) {
             stage_k(MK, slot, 0, kC);
         }
         int i = 0;
+        bool rdy = false;   // stage i+1 known complete (tested early during iteration i-1)
 #pragma unroll 1
         for (; i + 1 < nst; ++i) {
             int slN = slot;
             uint32_t phN = phase;
             advance(slN, phN);
-            wait_stage(slN, phN);
+            if (!LMO_EARLY_TEST || !rdy) wait_stage(slN, phN);
             stage_k(MK, slN, (i + 1) * kSub, kN);
+            if (LMO_EARLY_TEST) {   // non-blocking test of stage i+2: its latency hides under the V part
+                int slT = slN;
+                uint32_t phT = phN;
+                advance(slT, phT);
+                rdy = mbar_test(&wbar[slT], phT);
+            }
             stage_v(MK, slot, i * kSub, kC);
             slot = slN;
             phase = phN;
@@ -1312,14 +1347,21 @@ decode_attn_q4_kernel(const AttnArgs a) {
             else stage_k(GEN, slot, 0, kC);
         }
         int i = 0;
+        bool rdy = false;
         // steady state: contiguous hot loop (FULL K part of i+1, FULL V part of i)
 #pragma unroll 1
         for (; i + 1 < nfull; ++i) {
             int slN = slot;
             uint32_t phN = phase;
             advance(slN, phN);
-            wait_stage(slN, phN);
+            if (!LMO_EARLY_TEST || !rdy) wait_stage(slN, phN);
             stage_k(FULL, slN, (i + 1) * kSub, kN);
+            if (LMO_EARLY_TEST) {
+                int slT = slN;
+                uint32_t phT = phN;
+                advance(slT, phT);
+                rdy = mbar_test(&wbar[slT], phT);
+            }
             stage_v(FULL, slot, i * kSub, kC);
             slot = slN;
             phase = phN;

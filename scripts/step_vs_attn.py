@@ -18,23 +18,24 @@ for key in sys.argv[1:] or ["c4"]:
         for nm in ("k_meta", "v_meta"):
             c.field(nm).view(torch.int32).fill_(0x2C00BC00)
         caches.append(c)
-    q = torch.randn(w.batch, w.q_heads, w.head_dim, device='cuda').half()
-    kn = torch.randn(w.batch, w.kv_heads, 1, w.head_dim, device='cuda').half()
-    vn = torch.randn_like(kn)
+    # per-layer inputs (as in bench.py: not L2-resident when a layer's launch starts)
+    qs = [torch.randn(w.batch, w.q_heads, w.head_dim, device='cuda').half() for _ in range(nl)]
+    kns = [torch.randn(w.batch, w.kv_heads, 1, w.head_dim, device='cuda').half() for _ in range(nl)]
+    vns = [torch.randn_like(kns[0]) for _ in range(nl)]
     out = torch.empty(w.batch, w.q_heads, w.head_dim, device='cuda')
     ws = lmo.attention_workspace(w.batch, w.kv_heads, w.q_heads, w.head_dim)
     abis = [c.abi() for c in caches]
     st = torch.cuda.Stream()
     variants = {
-        "attn": lambda l: lmo.lmo_decode_attention_q4(caches[l], q, L, out=out, workspace=ws, abi=abis[l], stream=st),
-        "step_stable": lambda l: lmo.lmo_decode_step_q4(caches[l], kn, vn, q, L, out=out, workspace=ws, abi=abis[l],
+        "attn": lambda l: lmo.lmo_decode_attention_q4(caches[l], qs[l], L, out=out, workspace=ws, abi=abis[l], stream=st),
+        "step_stable": lambda l: lmo.lmo_decode_step_q4(caches[l], kns[l], vns[l], qs[l], L, out=out, workspace=ws, abi=abis[l],
                                                         flags=lmo.LMO_STEP_CACHE_STABLE, stream=st),
-        "step_plain": lambda l: lmo.lmo_decode_step_q4(caches[l], kn, vn, q, L, out=out, workspace=ws, abi=abis[l],
+        "step_plain": lambda l: lmo.lmo_decode_step_q4(caches[l], kns[l], vns[l], qs[l], L, out=out, workspace=ws, abi=abis[l],
                                                        stream=st),
-        "append+attn": lambda l: (lmo.lmo_kv_append_quant(caches[l], kn, vn, L - 1, abi=abis[l], stream=st),
-                                  lmo.lmo_decode_attention_q4(caches[l], q, L, out=out, workspace=ws, abi=abis[l],
+        "append+attn": lambda l: (lmo.lmo_kv_append_quant(caches[l], kns[l], vns[l], L - 1, abi=abis[l], stream=st),
+                                  lmo.lmo_decode_attention_q4(caches[l], qs[l], L, out=out, workspace=ws, abi=abis[l],
                                                               stream=st)),
-        "append": lambda l: lmo.lmo_kv_append_quant(caches[l], kn, vn, L - 1, abi=abis[l], stream=st),
+        "append": lambda l: lmo.lmo_kv_append_quant(caches[l], kns[l], vns[l], L - 1, abi=abis[l], stream=st),
     }
     res = {}
     for name, fn in variants.items():

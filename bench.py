@@ -632,11 +632,11 @@ def run_ours(args):
             p1.synchronize()
             pcie = max(pcie, 4 * (1 << 30) / (p0.elapsed_time(p1) / 1e3) / 1e9)
         del hb, db
-        h2d_step = nl * B * Hkv * (L - 1) * lmo.row_bytes(d)
+        h2d_step = nl * B * Hkv * (L & ~1) * lmo.row_bytes(d)      # old tokens as whole row pairs
         offload = {"value": sh.global_batch / (off_ms / 1e3), "unit": "tokens/s", "ms_per_step": off_ms,
                    "L": L, "ring_slots": 3, "host_bytes": host_bytes,
                    "h2d_bytes_per_step": h2d_step,
-                   "d2h_bytes_per_step": nl * B * Hkv * lmo.row_bytes(d),
+                   "d2h_bytes_per_step": nl * B * Hkv * 2 * lmo.row_bytes(d),   # the new token's row pair
                    "h2d_gbs": h2d_step / (off_ms / 1e3) / 1e9, "h2d_peak_gbs_measured": pcie,
                    "frac_of_h2d_peak": h2d_step / (off_ms / 1e3) / 1e9 / pcie,
                    "path": "pinned host q4 caches -> strided H2D (copy stream) -> fused step on a ring slot -> D2H of the new row"}

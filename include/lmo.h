@@ -89,10 +89,17 @@ lmo_status lmo_dequantize_groupwise(const uint8_t *codes, const lmo_qmeta *meta,
  * "compressed row" per (sequence, kv head, token slot):
  *   kv : [batch][kv_heads][capacity][row_bytes]        row_bytes = lmo_kv_row_bytes(head_dim)
  *   row: K codes (head_dim/2 B) | K meta (head_dim/64 lmo_qmeta) |
- *        V codes (head_dim/2 B) | V meta (head_dim/64 lmo_qmeta)
- * (144 B per token at head_dim 128, 72 B at 64).  Codes and meta are exactly
- * what lmo_quantize_groupwise(outer=1, n=head_dim, inner=1) produces for that
- * token's K (resp. V) row.  Token-major rows make a run of tokens of one
+ *        V area  (head_dim/2 B) | V meta (head_dim/64 lmo_qmeta)
+ * (144 B per token at head_dim 128, 72 B at 64).  K codes and both metas are
+ * exactly what lmo_quantize_groupwise(outer=1, n=head_dim, inner=1) produces for
+ * that token's K (resp. V) row.  The V codes of a token PAIR (slots 2p, 2p+1)
+ * are stored interleaved in 16-bit chunks of 4 dims: 32-bit word c of the pair =
+ * [token 2p chunk c (low half) | token 2p+1 chunk c (high half)], where chunk c
+ * holds the quantize_groupwise code bytes of dims 4c .. 4c+3; words 0 ..
+ * head_dim/8-1 fill the V area of row 2p, the rest that of row 2p+1.  (One word
+ * is then a tensor-core operand "(token, token) x 4 dims" without byte shuffles.)
+ * A token's V codes therefore live in both rows of its pair; appends write only
+ * the token's own 16-bit halves.  Token-major rows make a run of tokens of one
  * (sequence, kv head) a single contiguous span, i.e. one bulk copy.  Groups lie
  * along head_dim (reading 8), so every token's groups are
  * self-contained.  head_dim must be 64 or 128; capacity must be a multiple of
@@ -229,11 +236,13 @@ lmo_status lmo_offload_create(const lmo_kv_cache *shape, int32_t layers, uint8_t
 
 /* One decode step of all layers at length L = len (the new token goes to slot
  * len-1 of every layer's cache).  For each layer l:
- *   H2D   rows [0, len-1) of every (b, kvh) of host layer l -> ring slot
+ *   H2D   rows [0, len & ~1) of every (b, kvh) of host layer l -> ring slot
+ *         (the old tokens [0, len-1) as whole row pairs, see lmo_kv_cache)
  *         (one strided copy; waits until the slot's previous user is stored),
  *   A2-A4 lmo_decode_step_q4 on the slot with k_new/v_new/q of layer l
  *         (on compute_stream, after the H2D),
- *   D2H   row len-1 of every (b, kvh) of the slot -> host layer l.
+ *   D2H   the row pair of token len-1 (rows (len-1) & ~1 and +1) of every
+ *         (b, kvh) of the slot -> host layer l.
  * k_new, v_new : device [layers][B][Hkv][head_dim] fp16; q device
  * [layers][B][q_heads][head_dim] fp16; out device [layers][B][q_heads][head_dim]
  * (out_dtype).  Other arguments as lmo_decode_step_q4 (num_splits, workspace).

@@ -143,6 +143,19 @@ __device__ __forceinline__ uint2 quantize_group_lane4(const uint4 xa, const uint
     return make_uint2(codes8(xa, p), codes8(xb, p));
 }
 
+// ------------------------------------------------- KV cache row layout (lmo.h)
+// Token slot rows of `row` bytes: K codes (d/2) | K meta (d/64 words) | V area (d/2) |
+// V meta.  The V codes of a token PAIR (2p, 2p+1) are interleaved in 16-bit chunks of
+// 4 dims -- [A c | B c] per 32-bit word -- and the pair's 2 * d/2 bytes fill the V areas
+// of rows 2p (chunks 0 .. d/8-1) and 2p+1 (the rest): one 32-bit word is the MMA
+// operand "(token A, token B) x 4 dims" without any byte shuffling.
+// Store chunk c (codes of dims 4c .. 4c+3 of token `tok`) given the base of row tok & ~1.
+__device__ __forceinline__ void store_v_chunk(uint8_t *pair_row0, int d, int c, int tok, uint32_t v16) {
+    const int rb = d / 2, row = 2 * (rb + (d / 64) * 4), cpr = rb / 4;   // chunks per row
+    uint8_t *p = pair_row0 + (c / cpr) * row + rb + (d / 64) * 4 + 4 * (c % cpr) + 2 * (tok & 1);
+    *reinterpret_cast<uint16_t *>(p) = (uint16_t)v16;
+}
+
 // ------------------------------------------------------------- PTX wrappers
 __device__ __forceinline__ uint32_t smem_u32(const void *p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));

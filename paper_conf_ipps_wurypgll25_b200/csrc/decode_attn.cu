@@ -310,9 +310,9 @@ struct SegIter {
 };
 
 // ------------------------------------------------------------ fragments
-// Token order inside a 16-token block: MMA row r <-> token tperm(r) (a
-// bijection of 0..15 that halves shared-memory bank conflicts of the V loads).
-__device__ __forceinline__ int tperm(int r) { return r ^ ((r >> 1) & 1); }  // 0,1,3,2,4,5,7,6,...
+// Token order inside a 16-token block: MMA row r <-> token tperm(r).  With the
+// pair-interleaved V codes (round 2) the natural order is bank-conflict free.
+__device__ __forceinline__ int tperm(int r) { return r; }
 
 // Exact 4-bit codes as fp16 SUBNORMALS (no bias, no fp16 add):
 //   (x & 0x000F000F) reads the nibbles at bits 0-3 / 16-19 as c * 2^-24,
@@ -343,11 +343,10 @@ __device__ __forceinline__ void unpack_k(uint32_t w, uint32_t *u) {
     u[3] = s & 0x00F000F0u;
 }
 
-// V side: code words of two tokens A, B (same 8 dims) -> 8 half2 (A nib p, B nib p);
-// even p in the 2^-24 form, odd p in the 2^-20 form.
-__device__ __forceinline__ void unpack_v(uint32_t wa, uint32_t wb, uint32_t *j) {
-    const uint32_t lo = prmt(wa, wb, 0x5410u);   // [A.b0, A.b1, B.b0, B.b1]
-    const uint32_t hi = prmt(wa, wb, 0x7632u);   // [A.b2, A.b3, B.b2, B.b3]
+// V side: the cache stores the V codes of a token pair (2p, 2p+1) interleaved in 16-bit
+// chunks of 4 dims (include/lmo.h): lo = [A dims 8g..8g+3 | B same dims], hi = dims
+// 8g+4..8g+7 -> 8 half2 (A nib p, B nib p); even p in the 2^-24 form, odd p in 2^-20.
+__device__ __forceinline__ void unpack_v(uint32_t lo, uint32_t hi, uint32_t *j) {
     const uint32_t lo8 = shr8(lo), hi8 = shr8(hi);
     j[0] = lo & 0x000F000Fu;
     j[1] = lo & 0x00F000F0u;
@@ -374,6 +373,13 @@ __device__ __forceinline__ uint2 lds64(uint32_t a) {
     uint2 v;
     asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];\n" : "=r"(v.x), "=r"(v.y) : "r"(a));
     return v;
+}
+// two V code words (d = 128: 8-byte aligned; d = 64: the V area starts at byte 36 of a
+// 72-byte row, 4-byte alignment only)
+template <int NG>
+__device__ __forceinline__ uint2 load_v2(uint32_t a) {
+    if constexpr (NG == 2) return lds64(a);
+    else return make_uint2(lds32(a), lds32(a + 4));
 }
 // the NG meta words of one row (NG = 1: 4-byte aligned only)
 template <int NG>
@@ -612,7 +618,8 @@ decode_attn_q4_kernel(const AttnArgs a) {
     // bump; segment transitions (work-map arithmetic) run out of line.
     auto issue = [&](int slot) {
         const int n = min(kStageTok, ctl.pend - ctl.ptok);
-        const uint32_t bytes = (n * GG::ROW + 15) & ~15;          // cap % 16 == 0: in bounds
+        // whole token pairs (a pair's V codes span both rows); cap % 16 == 0 keeps it in bounds
+        const uint32_t bytes = ((n + 1) & ~1) * GG::ROW;
         mbar_arrive_expect_tx(&wbar[slot], bytes);
         bulk_g2s(wring + slot * GG::STAGE, ctl.psrc, bytes, &wbar[slot], pol);
         ctl.psrc += kStageTok * GG::ROW;
@@ -809,7 +816,14 @@ decode_attn_q4_kernel(const AttnArgs a) {
                 if (lane_ok && Lb >= 1) {
                     uint8_t *row = const_cast<uint8_t *>(a.kv) + ((int64_t)p * a.cap + Lb - 1) * GG::ROW +
                                    kvsel * (GG::RB + GG::MB);
-                    reinterpret_cast<uint32_t *>(row + grp8 * 32)[lane8] = w;
+                    if (kvsel == 0) {
+                        reinterpret_cast<uint32_t *>(row + grp8 * 32)[lane8] = w;
+                    } else {                      // pair-interleaved V codes: two 16-bit chunks
+                        uint8_t *pr = const_cast<uint8_t *>(a.kv) + ((int64_t)p * a.cap + ((Lb - 1) & ~1)) * GG::ROW;
+                        const int c = 16 * grp8 + 2 * lane8;
+                        store_v_chunk(pr, D, c, Lb - 1, w & 0xFFFFu);
+                        store_v_chunk(pr, D, c + 1, Lb - 1, w >> 16);
+                    }
                     if (lane8 == 0) reinterpret_cast<uint32_t *>(row + GG::RB)[grp8] = mw;
                 }
             }
@@ -876,8 +890,10 @@ decode_attn_q4_kernel(const AttnArgs a) {
     const uint32_t offK0 = ring_u32 + tk0 * GG::ROW + 8 * t;
     const uint32_t offKm0 = ring_u32 + tk0 * GG::ROW + GG::OKM;
     const uint32_t offVm0 = ring_u32 + tk0 * GG::ROW + GG::OVM;
-    const uint32_t offVa0 = ring_u32 + tperm(2 * t) * GG::ROW + GG::OVC + 4 * g;
-    const uint32_t offVb0 = ring_u32 + tperm(2 * t + 1) * GG::ROW + GG::OVC + 4 * g;
+    // V codes of token pair (2t, 2t+1), dims 8g..8g+7 of group grp: chunk c = (grp*64 + 8g)/4
+    // lives in row 2t + c / (RB/4), word c % (RB/4) (d = 128: row 2t + grp, word 2g)
+    const uint32_t offV0 = ring_u32 + (2 * t + (NG == 2 ? 0 : (g >> 2))) * GG::ROW + GG::OVC +
+                           8 * (NG == 2 ? g : (g & 3));
     constexpr int dK1 = 8 * GG::ROW;   // token row +8
     constexpr int dM1 = 8 * GG::ROW;
     constexpr int dSC = kBlk * GG::ROW; // sub-block stride
@@ -1176,13 +1192,11 @@ decode_attn_q4_kernel(const AttnArgs a) {
                         for (int grp = 0; grp < NG; ++grp) {
                             const uint32_t sel = grp == 0 ? 0x5410u : 0x7632u;
                             const uint32_t bp0 = prmt(x0, x1, sel), bp1 = prmt(x2, x3, sel);
-                            const uint32_t wa0 = lds32(ss + offVa0 + grp * 32);
-                            const uint32_t wb0 = lds32(ss + offVb0 + grp * 32);
-                            const uint32_t wa1 = lds32(ss + offVa0 + dK1 + grp * 32);
-                            const uint32_t wb1 = lds32(ss + offVb0 + dK1 + grp * 32);
+                            const uint2 v0 = load_v2<NG>(ss + offV0 + grp * GG::ROW);
+                            const uint2 v1 = load_v2<NG>(ss + offV0 + dK1 + grp * GG::ROW);
                             uint32_t j0[8], j1[8];
-                            unpack_v(wa0, wb0, j0);
-                            unpack_v(wa1, wb1, j1);
+                            unpack_v(v0.x, v0.y, j0);
+                            unpack_v(v1.x, v1.y, j1);
 #pragma unroll
                             for (int mbl = 0; mbl < 4; ++mbl)
                                 mma_16816(acc[grp * 4 + mbl], j0[2 * mbl], j0[2 * mbl + 1], j1[2 * mbl],
@@ -1273,13 +1287,11 @@ decode_attn_q4_kernel(const AttnArgs a) {
                         // P^T: (token row, heads 2t..2t+1) -> transpose -> (head g, tokens 2t..2t+1)
                         const uint32_t bp0 = movmatrix_t(pack_half2(p[0][0] * f0.y, p[0][1] * f0.y));
                         const uint32_t bp1 = movmatrix_t(pack_half2(p[1][0] * f1.y, p[1][1] * f1.y));
-                        const uint32_t wa0 = lds32(ss + offVa0 + grp * 32);
-                        const uint32_t wb0 = lds32(ss + offVb0 + grp * 32);
-                        const uint32_t wa1 = lds32(ss + offVa0 + dK1 + grp * 32);
-                        const uint32_t wb1 = lds32(ss + offVb0 + dK1 + grp * 32);
+                        const uint2 v0 = load_v2<NG>(ss + offV0 + grp * GG::ROW);
+                        const uint2 v1 = load_v2<NG>(ss + offV0 + dK1 + grp * GG::ROW);
                         uint32_t j0[8], j1[8];
-                        unpack_v(wa0, wb0, j0);
-                        unpack_v(wa1, wb1, j1);
+                        unpack_v(v0.x, v0.y, j0);
+                        unpack_v(v1.x, v1.y, j1);
 #pragma unroll
                         for (int mbl = 0; mbl < 4; ++mbl)
                             mma_16816(acc[grp * 4 + mbl], j0[2 * mbl], j0[2 * mbl + 1], j1[2 * mbl],

@@ -6,7 +6,7 @@
 // (cudaMemcpy2DAsync: B*Hkv rows of (L-1)*row bytes, pitch cap*row) on a
 // dedicated H2D stream into a device ring slot; the fused decode step
 // (A2+A3+A4, decode_attn.cu) runs on the slot on the caller's stream; the new
-// token's row goes back with one strided D2H on a second copy stream (the two
+// token's row pair (V codes are pair-interleaved) goes back with one strided D2H on a second copy stream (the two
 // PCIe directions overlap).  Per-slot events order slot reuse.  All
 // enqueue-only; no device allocation.
 #include <new>
@@ -136,10 +136,12 @@ lmo_status lmo_offload_decode_step(lmo_offload_t x, const void *k_new, const voi
         const int s = l % x->slots;
         uint8_t *slot = x->ring + (size_t)s * x->layer_bytes;
         uint8_t *host = x->host + (size_t)l * x->layer_bytes;
-        // load_cache: old-token rows [0, len-1) of every (b, kvh)
+        // load_cache: the old tokens [0, len-1) of every (b, kvh), as whole token pairs
+        // (rows [0, len & ~1): an old token's pair partner row carries half its V codes)
         cudaError_t e = cudaStreamWaitEvent(x->h2d, x->freed[s], 0);
-        if (e == cudaSuccess && len > 1)
-            e = cudaMemcpy2DAsync(slot, pitch, host, pitch, (size_t)(len - 1) * x->row, pairs,
+        const size_t nrows = (size_t)(len & ~1);
+        if (e == cudaSuccess && nrows > 0)
+            e = cudaMemcpy2DAsync(slot, pitch, host, pitch, nrows * x->row, pairs,
                                   cudaMemcpyHostToDevice, x->h2d);
         if (e == cudaSuccess) e = cudaEventRecord(x->loaded[s], x->h2d);
         if (e == cudaSuccess) e = cudaStreamWaitEvent(cs, x->loaded[s], 0);
@@ -154,12 +156,13 @@ lmo_status lmo_offload_decode_step(lmo_offload_t x, const void *k_new, const voi
             num_splits, static_cast<uint8_t *>(out) + l * o_layer, out_dtype, workspace,
             workspace_bytes, 0u, cs);
         if (st != LMO_OK) return st;
-        // store_cache: the new token's row back to host memory
+        // store_cache: the new token back to host memory -- the two rows of its token pair
+        // (the pair's V codes are interleaved across both rows, include/lmo.h)
         e = cudaEventRecord(x->computed[s], cs);
         if (e == cudaSuccess) e = cudaStreamWaitEvent(x->d2h, x->computed[s], 0);
+        const size_t r0 = (size_t)((len - 1) & ~1);
         if (e == cudaSuccess)
-            e = cudaMemcpy2DAsync(host + (size_t)(len - 1) * x->row, pitch,
-                                  slot + (size_t)(len - 1) * x->row, pitch, x->row, pairs,
+            e = cudaMemcpy2DAsync(host + r0 * x->row, pitch, slot + r0 * x->row, pitch, 2 * x->row, pairs,
                                   cudaMemcpyDeviceToHost, x->d2h);
         if (e == cudaSuccess) e = cudaEventRecord(x->freed[s], x->d2h);
         if (e != cudaSuccess) return LMO_ERR_CUDA;

@@ -122,10 +122,19 @@ __global__ void __launch_bounds__(256) kv_append_kernel(lmo_kv_cache cache,
         if (valid) {
             const int64_t slot = (int64_t)bh * cache.capacity + pos + t;
             uint8_t *row = cache.kv + slot * ROW + kv * (RB + MB);
-            // the V half of a d=64 row starts at byte 36: only 4-byte alignment holds
-            uint32_t *dst = reinterpret_cast<uint32_t *>(row + grp * 32 + lane4 * 8);
-            dst[0] = w.x;
-            dst[1] = w.y;
+            if (kv == 0) {
+                uint32_t *dst = reinterpret_cast<uint32_t *>(row + grp * 32 + lane4 * 8);
+                dst[0] = w.x;
+                dst[1] = w.y;
+            } else {   // V codes: pair-interleaved 16-bit chunks (common.cuh, include/lmo.h)
+                const int tok = pos + t;
+                uint8_t *pr = cache.kv + ((int64_t)bh * cache.capacity + (tok & ~1)) * ROW;
+                const int c = 16 * grp + 4 * lane4;
+                store_v_chunk(pr, d, c, tok, w.x & 0xFFFFu);
+                store_v_chunk(pr, d, c + 1, tok, w.x >> 16);
+                store_v_chunk(pr, d, c + 2, tok, w.y & 0xFFFFu);
+                store_v_chunk(pr, d, c + 3, tok, w.y >> 16);
+            }
             if (lane4 == 0) reinterpret_cast<uint32_t *>(row + RB)[grp] = mw;
         }
     }

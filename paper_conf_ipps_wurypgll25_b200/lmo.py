@@ -225,24 +225,36 @@ class KVCache:
     def nbytes(self) -> int:
         return self.kv.numel()
 
-    # field views (strided): codes [B][Hkv][cap][d/2] u8, meta [B][Hkv][cap][d/64] as int32 bytes
+    # field views (strided): K codes [B][Hkv][cap][d/2] u8, meta [B][Hkv][cap][d/64] as
+    # int32 bytes.  The V codes are pair-interleaved (include/lmo.h): no per-token view.
     def field(self, name: str) -> torch.Tensor:
         rb, mb = self.head_dim // 2, 4 * (self.head_dim // GROUP)
-        off = {"k_codes": (0, rb), "k_meta": (rb, mb), "v_codes": (rb + mb, rb),
-               "v_meta": (2 * rb + mb, mb)}[name]
+        if name == "v_codes":
+            raise ValueError("V codes are stored pair-interleaved; use to_host_fields()")
+        off = {"k_codes": (0, rb), "k_meta": (rb, mb), "v_meta": (2 * rb + mb, mb)}[name]
         return self.kv[..., off[0]:off[0] + off[1]]
 
     def to_host_fields(self):
         """Copy to host as the oracle's field arrays: codes uint8 [B][Hkv][cap][d/2],
-        meta uint16 [B][Hkv][cap][d/64][2] ({min, scale} bit patterns)."""
+        meta uint16 [B][Hkv][cap][d/64][2] ({min, scale} bit patterns).  The V codes are
+        de-interleaved from the pair layout: the V areas of rows 2p, 2p+1 hold the 16-bit
+        4-dim chunks of tokens 2p (low half of each word) and 2p+1 (high half)."""
         import numpy as np
         kv = self.kv.cpu().numpy()
         rb, ng = self.head_dim // 2, self.head_dim // GROUP
         out = {}
         for name in ("k_codes", "k_meta", "v_codes", "v_meta"):
             off = {"k_codes": 0, "k_meta": rb, "v_codes": rb + 4 * ng, "v_meta": 2 * rb + 4 * ng}[name]
-            if name.endswith("codes"):
+            if name == "k_codes":
                 out[name] = np.ascontiguousarray(kv[..., off:off + rb])
+            elif name == "v_codes":
+                B, H, cap = kv.shape[:3]
+                area = np.ascontiguousarray(kv[..., off:off + rb]).reshape(B, H, cap // 2, 2 * rb)
+                w = area.view(np.uint16)                               # [B][H][pairs][d/4 words x 2 halves]
+                v = np.empty((B, H, cap // 2, 2, rb), np.uint8)
+                v[:, :, :, 0] = np.ascontiguousarray(w[..., 0::2]).view(np.uint8)
+                v[:, :, :, 1] = np.ascontiguousarray(w[..., 1::2]).view(np.uint8)
+                out[name] = v.reshape(B, H, cap, rb)
             else:
                 m = np.ascontiguousarray(kv[..., off:off + 4 * ng])
                 out[name] = m.view(np.uint16).reshape(*m.shape[:-1], ng, 2)

@@ -38,7 +38,8 @@ def test_offload_matches_resident(lmo, slots, G, d, nl):
         lmo.lmo_gen_fill_f16(kall[l], seed, I.STREAM_K, l, 0, 0, 0)
         lmo.lmo_gen_fill_f16(vall[l], seed, I.STREAM_V, l, 0, 0, 0)
         lmo.lmo_kv_append_quant(res[l], kall[l, :, :, :s0].contiguous(), vall[l, :, :, :s0].contiguous(), 0)
-        off.host_layer(l)[:, :, :s0].copy_(res[l].kv[:, :, :s0].cpu())
+        s2 = s0 + (s0 & 1)                        # whole token pairs (V codes span both rows)
+        off.host_layer(l)[:, :, :s2].copy_(res[l].kv[:, :, :s2].cpu())
     torch.cuda.synchronize()
     ws = lmo.attention_workspace(B, Hkv, Hq, d)
     for t in range(1, steps + 1):
@@ -55,8 +56,11 @@ def test_offload_matches_resident(lmo, slots, G, d, nl):
         torch.cuda.synchronize()
         assert torch.equal(got, want), f"step {t}"
     L = s0 + steps
-    for l in range(nl):
-        assert torch.equal(off.host_layer(l)[:, :, :L], res[l].kv[:, :, :L].cpu()), l
+    for l in range(nl):   # every field of tokens [0, L), V codes de-interleaved from the row pairs
+        hv = lmo.KVCache(off.host_layer(l), B, Hkv, off.capacity, d).to_host_fields()
+        rv = res[l].to_host_fields()
+        for key in rv:
+            assert np.array_equal(hv[key][:, :, :L], rv[key][:, :, :L]), (l, key)
     # and the last step of layer 0 against the oracle (host cache bytes -> oracle fields)
     host = oracle.new_cache(B, Hkv, res[0].capacity, d)
     oracle.kv_append_quant(host, kall[0, :, :, :L].cpu().numpy(), vall[0, :, :, :L].cpu().numpy(), 0)

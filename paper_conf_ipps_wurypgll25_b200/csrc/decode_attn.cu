@@ -827,7 +827,9 @@ decode_attn_q4_kernel(const AttnArgs a) {
                     if (lane8 == 0) reinterpret_cast<uint32_t *>(row + GG::RB)[grp8] = mw;
                 }
             }
+#ifndef LMO_NO_APPEND_FENCE
             asm volatile("fence.proxy.async.global;\n" ::: "memory");
+#endif
         }
         __syncwarp();
     };
@@ -1483,7 +1485,70 @@ decode_attn_q4_kernel(const AttnArgs a) {
             }
         }
         const bool full = SCH == 1 || (SCH == 0 && (sd.blk0 == 0) && (sd.sn == sd.nb) && wms.T <= 1);
-        if (SCH == 2 || (SCH == 0 && wms.T > 1)) {
+        if (SCH == 2 && wms.T == 2 && sd.v + wms.n_teams >= a.B * a.Hkv) {
+            // ---- pair team of 2, the team's LAST pair (the only pair when teams outnumber
+            // pairs -- the T = 2 regime): A4 on chip.  Rank 1's producer has issued nothing
+            // beyond this segment and every issued stage is consumed, so its TMA ring is idle:
+            // rank 1 writes its partial (numerators, m, l -- in the SAME lane layout) there,
+            // arrives on a named barrier; rank 0 syncs, merges in registers and stores.  No L2
+            // round trip, no atomics, no extra shared memory.
+            const int ti = warp >> 1, rank = warp & 1;
+            const uint32_t bar_full = 1 + ti;
+            float *part = reinterpret_cast<float *>(ring + (size_t)(2 * ti + 1) * kStages * GG::STAGE);
+            if (rank == 1) {
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                    const int h = 2 * t + e;
+                    if (h < a.G) {
+                        float *ph = part + h * (D + 4);             // (16-B aligned head records)
+#pragma unroll
+                        for (int grp = 0; grp < NG; ++grp) {
+                            float4 *r4 = reinterpret_cast<float4 *>(ph + grp * 64 + 8 * g);
+                            r4[0] = make_float4(vo[e][grp][0], vo[e][grp][1], vo[e][grp][2], vo[e][grp][3]);
+                            r4[1] = make_float4(vo[e][grp][4], vo[e][grp][5], vo[e][grp][6], vo[e][grp][7]);
+                        }
+                        if (g == 0) {
+                            ph[D] = m_run[e] == NEG_INF ? NEG_INF : mE[e];
+                            ph[D + 1] = lt[e];
+                        }
+                    }
+                }
+                asm volatile("bar.arrive %0, 64;\n" ::"r"(bar_full) : "memory");
+            } else {
+                asm volatile("bar.sync %0, 64;\n" ::"r"(bar_full) : "memory");
+                float o1[2][NG][8], m1[2], l1[2];
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                    const float *ph = part + min(2 * t + e, a.G - 1) * (D + 4);
+#pragma unroll
+                    for (int grp = 0; grp < NG; ++grp) {
+                        const float4 *r4 = reinterpret_cast<const float4 *>(ph + grp * 64 + 8 * g);
+                        const float4 x0 = r4[0], x1 = r4[1];
+                        o1[e][grp][0] = x0.x; o1[e][grp][1] = x0.y; o1[e][grp][2] = x0.z; o1[e][grp][3] = x0.w;
+                        o1[e][grp][4] = x1.x; o1[e][grp][5] = x1.y; o1[e][grp][6] = x1.z; o1[e][grp][7] = x1.w;
+                    }
+                    m1[e] = ph[D];
+                    l1[e] = ph[D + 1];
+                }
+#pragma unroll
+                for (int e = 0; e < 2; ++e) {
+                    const int h = 2 * t + e;
+                    const float m0 = m_run[e] == NEG_INF ? NEG_INF : mE[e];
+                    const float M = fmaxf(m0, m1[e]);
+                    if (h >= a.G || M == NEG_INF) continue;      // (empty sequence: zero row written)
+                    const float w0 = fast_exp2(m0 - M), w1 = fast_exp2(m1[e] - M);
+                    const float il = 1.f / fmaf(lt[e], w0, l1[e] * w1);
+#pragma unroll
+                    for (int grp = 0; grp < NG; ++grp) {
+                        float o[8];
+#pragma unroll
+                        for (int i = 0; i < 8; ++i) o[i] = fmaf(vo[e][grp][i], w0, o1[e][grp][i] * w1) * il;
+                        store_row8<D>(a, rowbase + h, grp * 64 + 8 * g, o);
+                    }
+                }
+            }
+            ++team_k;
+        } else if (SCH == 2 || (SCH == 0 && wms.T > 1)) {
             // ---- pair team: partials through L2 scratch, named barrier, rank 0 merges
             const int T = wms.T;
             const int64_t myslot = 2 * (int64_t)gw + (team_k & 1);
@@ -1796,8 +1861,12 @@ static size_t smem_bytes(int B_prefix) {
     return bars_bytes<NW>() + (size_t)NW * kStages * Geo<D>::STAGE + (B_prefix > 0 ? (B_prefix + 1) * sizeof(int) : 0);
 }
 
+
 // SM teams: one CTA of kSmWarps warps per SM (the ring fills the SM's shared memory)
-constexpr int kSmWarps = 16;
+#ifndef LMO_SM_WARPS
+#define LMO_SM_WARPS 16
+#endif
+constexpr int kSmWarps = LMO_SM_WARPS;
 template <int D>
 static bool sm_team_ok() {
     static std::atomic<int> ok[64];   // 0 unknown, 1 yes, 2 no (idempotent once-per-device probe)

@@ -10,7 +10,7 @@ pids=()
 while [ $# -ge 2 ]; do
   name=$1; defs=$2; shift 2
   /usr/local/cuda/bin/nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 \
-    -Xcompiler -fPIC,-O2 --shared -cudart static $defs -I include -I $PKG/csrc \
+    -Xcompiler -fPIC,-O2 -Xptxas -v --shared -cudart static $defs -I include -I $PKG/csrc \
     -o build/variants/$name.so $PKG/csrc/*.cu > build/variants/$name.log 2>&1 &
   pids+=($!)
 done

@@ -23,13 +23,15 @@ for key in sys.argv[1:] or ["c4"]:
     kns = [torch.randn(w.batch, w.kv_heads, 1, w.head_dim, device='cuda').half() for _ in range(nl)]
     vns = [torch.randn_like(kns[0]) for _ in range(nl)]
     out = torch.empty(w.batch, w.q_heads, w.head_dim, device='cuda')
-    ws = lmo.attention_workspace(w.batch, w.kv_heads, w.q_heads, w.head_dim)
+    ws = lmo.attention_workspace(w.batch, w.kv_heads, w.q_heads, w.head_dim, int(os.environ.get("SPLITS", "0")))
     abis = [c.abi() for c in caches]
     st = torch.cuda.Stream()
+    ns = int(os.environ.get("SPLITS", "0"))
     variants = {
-        "attn": lambda l: lmo.lmo_decode_attention_q4(caches[l], qs[l], L, out=out, workspace=ws, abi=abis[l], stream=st),
+        "attn": lambda l: lmo.lmo_decode_attention_q4(caches[l], qs[l], L, out=out, workspace=ws, abi=abis[l], stream=st,
+                                                   num_splits=ns),
         "step_stable": lambda l: lmo.lmo_decode_step_q4(caches[l], kns[l], vns[l], qs[l], L, out=out, workspace=ws, abi=abis[l],
-                                                        flags=lmo.LMO_STEP_CACHE_STABLE, stream=st),
+                                                        flags=lmo.LMO_STEP_CACHE_STABLE, stream=st, num_splits=ns),
         "step_plain": lambda l: lmo.lmo_decode_step_q4(caches[l], kns[l], vns[l], qs[l], L, out=out, workspace=ws, abi=abis[l],
                                                        stream=st),
         "append+attn": lambda l: (lmo.lmo_kv_append_quant(caches[l], kns[l], vns[l], L - 1, abi=abis[l], stream=st),

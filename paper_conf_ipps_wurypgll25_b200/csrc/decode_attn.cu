@@ -63,6 +63,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_GQA_VOTE
 #define LMO_GQA_VOTE 1   // GQA FULL stages: rescale only when a running max moved (one vote)
 #endif
+#ifndef LMO_TEAM_RING_ONLY
+#define LMO_TEAM_RING_ONLY 1   // the T > 1 instance merges only on chip: launched only when every
+#endif                         // team has at most one pair (else the generic instance, L2 merge)
 #ifndef LMO_EARLY_TEST
 #define LMO_EARLY_TEST 0   // non-blocking mbarrier test of stage i+2 during iteration i
 #endif
@@ -1485,17 +1488,21 @@ decode_attn_q4_kernel(const AttnArgs a) {
             }
         }
         const bool full = SCH == 1 || (SCH == 0 && (sd.blk0 == 0) && (sd.sn == sd.nb) && wms.T <= 1);
-        if (SCH == 2 && wms.T == 2 && sd.v + wms.n_teams >= a.B * a.Hkv) {
-            // ---- pair team of 2, the team's LAST pair (the only pair when teams outnumber
-            // pairs -- the T = 2 regime): A4 on chip.  Rank 1's producer has issued nothing
-            // beyond this segment and every issued stage is consumed, so its TMA ring is idle:
-            // rank 1 writes its partial (numerators, m, l -- in the SAME lane layout) there,
-            // arrives on a named barrier; rank 0 syncs, merges in registers and stores.  No L2
-            // round trip, no atomics, no extra shared memory.
-            const int ti = warp >> 1, rank = warp & 1;
-            const uint32_t bar_full = 1 + ti;
-            float *part = reinterpret_cast<float *>(ring + (size_t)(2 * ti + 1) * kStages * GG::STAGE);
-            if (rank == 1) {
+        if (SCH == 2 && sd.v + wms.n_teams >= a.B * a.Hkv) {
+            // ---- pair team (T = 2 or 4), the team's LAST pair (the only pair when teams
+            // outnumber pairs -- the regime teams are chosen for): A4 on chip.  The producers of
+            // ranks 1..T-1 have issued nothing beyond this segment and every issued stage is
+            // consumed, so their TMA rings are idle: each writes its partial (numerators, m, l
+            // -- in the SAME lane layout) into its own ring and arrives on a named barrier; rank
+            // 0 syncs, merges in registers and stores.  No L2 round trip, no atomics, no extra
+            // shared memory.
+            const int T = wms.T, ti = warp / T, rank = warp - ti * T;
+            const uint32_t bar_full = 1 + ti, bar_n = 32 * T;
+            auto part_of = [&](int r) {
+                return reinterpret_cast<float *>(ring + (size_t)(ti * T + r) * kStages * GG::STAGE);
+            };
+            if (rank != 0) {
+                float *part = part_of(rank);
 #pragma unroll
                 for (int e = 0; e < 2; ++e) {
                     const int h = 2 * t + e;
@@ -1513,42 +1520,49 @@ decode_attn_q4_kernel(const AttnArgs a) {
                         }
                     }
                 }
-                asm volatile("bar.arrive %0, 64;\n" ::"r"(bar_full) : "memory");
+                asm volatile("bar.arrive %0, %1;\n" ::"r"(bar_full), "r"(bar_n) : "memory");
             } else {
-                asm volatile("bar.sync %0, 64;\n" ::"r"(bar_full) : "memory");
-                float o1[2][NG][8], m1[2], l1[2];
-#pragma unroll
-                for (int e = 0; e < 2; ++e) {
-                    const float *ph = part + min(2 * t + e, a.G - 1) * (D + 4);
-#pragma unroll
-                    for (int grp = 0; grp < NG; ++grp) {
-                        const float4 *r4 = reinterpret_cast<const float4 *>(ph + grp * 64 + 8 * g);
-                        const float4 x0 = r4[0], x1 = r4[1];
-                        o1[e][grp][0] = x0.x; o1[e][grp][1] = x0.y; o1[e][grp][2] = x0.z; o1[e][grp][3] = x0.w;
-                        o1[e][grp][4] = x1.x; o1[e][grp][5] = x1.y; o1[e][grp][6] = x1.z; o1[e][grp][7] = x1.w;
-                    }
-                    m1[e] = ph[D];
-                    l1[e] = ph[D + 1];
-                }
+                asm volatile("bar.sync %0, %1;\n" ::"r"(bar_full), "r"(bar_n) : "memory");
 #pragma unroll
                 for (int e = 0; e < 2; ++e) {
                     const int h = 2 * t + e;
+                    const int hc = min(h, a.G - 1);
                     const float m0 = m_run[e] == NEG_INF ? NEG_INF : mE[e];
-                    const float M = fmaxf(m0, m1[e]);
+                    float M = m0;
+                    for (int r = 1; r < T; ++r) M = fmaxf(M, part_of(r)[hc * (D + 4) + D]);
                     if (h >= a.G || M == NEG_INF) continue;      // (empty sequence: zero row written)
-                    const float w0 = fast_exp2(m0 - M), w1 = fast_exp2(m1[e] - M);
-                    const float il = 1.f / fmaf(lt[e], w0, l1[e] * w1);
+                    const float w0 = fast_exp2(m0 - M);
+                    float l = lt[e] * w0;
+                    float o[NG][8];
+#pragma unroll
+                    for (int grp = 0; grp < NG; ++grp)
+#pragma unroll
+                        for (int i = 0; i < 8; ++i) o[grp][i] = vo[e][grp][i] * w0;
+                    for (int r = 1; r < T; ++r) {
+                        const float *ph = part_of(r) + hc * (D + 4);
+                        const float wr = fast_exp2(ph[D] - M);
+                        l = fmaf(ph[D + 1], wr, l);
+#pragma unroll
+                        for (int grp = 0; grp < NG; ++grp) {
+                            const float4 *r4 = reinterpret_cast<const float4 *>(ph + grp * 64 + 8 * g);
+                            const float4 x0 = r4[0], x1 = r4[1];
+                            o[grp][0] = fmaf(x0.x, wr, o[grp][0]); o[grp][1] = fmaf(x0.y, wr, o[grp][1]);
+                            o[grp][2] = fmaf(x0.z, wr, o[grp][2]); o[grp][3] = fmaf(x0.w, wr, o[grp][3]);
+                            o[grp][4] = fmaf(x1.x, wr, o[grp][4]); o[grp][5] = fmaf(x1.y, wr, o[grp][5]);
+                            o[grp][6] = fmaf(x1.z, wr, o[grp][6]); o[grp][7] = fmaf(x1.w, wr, o[grp][7]);
+                        }
+                    }
+                    const float il = 1.f / l;
 #pragma unroll
                     for (int grp = 0; grp < NG; ++grp) {
-                        float o[8];
 #pragma unroll
-                        for (int i = 0; i < 8; ++i) o[i] = fmaf(vo[e][grp][i], w0, o1[e][grp][i] * w1) * il;
-                        store_row8<D>(a, rowbase + h, grp * 64 + 8 * g, o);
+                        for (int i = 0; i < 8; ++i) o[grp][i] *= il;
+                        store_row8<D>(a, rowbase + h, grp * 64 + 8 * g, o[grp]);
                     }
                 }
             }
             ++team_k;
-        } else if (SCH == 2 || (SCH == 0 && wms.T > 1)) {
+        } else if ((SCH == 2 && !LMO_TEAM_RING_ONLY) || (SCH == 0 && wms.T > 1)) {
             // ---- pair team: partials through L2 scratch, named barrier, rank 0 merges
             const int T = wms.T;
             const int64_t myslot = 2 * (int64_t)gw + (team_k & 1);
@@ -2030,6 +2044,7 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     int64_t want_warps;
     if (a.team) {
         want_warps = (int64_t)max_ctas * kWarps;          // all CTAs; idle teams exit at once
+
 #ifdef LMO_EXPERIMENTS
         static const char *tight = getenv("LMO_ATTN_TIGHT");   // experiments: grid = teams
         if (tight && tight[0] == '1') want_warps = pairs * a.team;
@@ -2092,7 +2107,7 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false, kWarps, 1>, a))
                     : (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, true, kWarps, 1>, a)
                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, false, kWarps, 1>, a));
-    else if (a.team > 1 && !LMO_NO_SCH)
+    else if (a.team > 1 && !LMO_NO_SCH && pairs <= (int64_t)a.wm.n_teams)
         e = D == 64 ? (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, true, kWarps, 2>, a)
                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false, kWarps, 2>, a))
                     : (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, true, kWarps, 2>, a)

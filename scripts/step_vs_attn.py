@@ -7,8 +7,11 @@ import torch
 from paper_conf_ipps_wurypgll25_b200 import lmo
 from paper_conf_ipps_wurypgll25_b200.configs import CONFIGS
 
+import dataclasses
 for key in sys.argv[1:] or ["c4"]:
-    w = CONFIGS[key]
+    w = CONFIGS[key.split(":")[0]]
+    if ":" in key:                                   # c4:8 -> the config at batch 8 (strong-scaling shard)
+        w = dataclasses.replace(w, batch=int(key.split(":")[1]))
     L = w.prompt + w.gen // 2
     nl = max(4, min(64, int(6.0e9 // (w.batch * w.kv_heads * w.capacity * 144))))
     caches = []

@@ -63,6 +63,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_GQA_VOTE
 #define LMO_GQA_VOTE 1   // GQA FULL stages: rescale only when a running max moved (one vote)
 #endif
+#ifndef LMO_SMALL_CTAS_PER_SM
+#define LMO_SMALL_CTAS_PER_SM 2   // small-batch team launches: resident CTAs per SM (0: no cap); measured
+#endif                            // better than a 3-per-SM cap for 256-CTA launches
 #ifndef LMO_TEAM_RING_ONLY
 #define LMO_TEAM_RING_ONLY 1   // the T > 1 instance merges only on chip: launched only when every
 #endif                         // team has at most one pair (else the generic instance, L2 merge)
@@ -1913,8 +1916,8 @@ static int ctas_per_sm(int B_prefix, bool mha) {   // (MHA and GQA instances dif
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kWarps, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
         cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
-        cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kWarps, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
-        cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<D, true, kWarps, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<D, false, kWarps, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
         int n = 0;
         const size_t smem = smem_bytes<D>(mode ? kMaxBatchSmem : 0);
         // the least occupancy over the schedule instances of this variant (same bound; SCH 0 is the largest)
@@ -2055,8 +2058,28 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
         const int64_t N = pairs * nbu;
         want_warps = num_splits > 0 ? pairs * num_splits : N;
     }
+    // Small batches (teams of T > 1, every team at most one pair, <= 2 working CTAs per SM):
+    // cap the resident CTAs at 2 per SM (padded shared memory).  With 4 per SM and
+    // programmatic dependent launch, the next launch's low CTA ids -- the ones with work --
+    // land 2-4 to an SM in the slots the previous launch's idle CTAs free, leaving other SMs
+    // idle (timeline: 128 working CTAs on 70 SMs); with 2 per SM a launch with <= 148
+    // working CTAs gets one SM each and a landing slot for the next launch on every SM
+    // (c5 at batch 16: 21.7 -> 14.4 us, c2 at batch 4: 10.9 -> 7.7 us).
+    size_t pad_smem = 0;
+    int64_t cap_ctas = max_ctas;
+    const int64_t need_ctas = (pairs * a.team + kWarps - 1) / kWarps;
+    const int per_sm_cap = LMO_SMALL_CTAS_PER_SM;
+    const bool small = per_sm_cap > 0 && a.team > 1 && pairs <= (int64_t)max_ctas * kWarps / a.team &&
+                       need_ctas <= (int64_t)device_sm_count() * per_sm_cap && per_sm_cap < max_ctas / device_sm_count();
+    if (small) {
+        cap_ctas = (int64_t)device_sm_count() * per_sm_cap;
+        const size_t per_sm = 228 * 1024, want = per_sm / per_sm_cap - 2048;
+        const size_t base = D == 64 ? smem_bytes<64>(Bp) : smem_bytes<128>(Bp);
+        if (want > base) pad_smem = want - base;
+        if (want_warps > cap_ctas * kWarps) want_warps = cap_ctas * kWarps;
+    }
     int64_t ctas = (want_warps + kWarps - 1) / kWarps;
-    if (ctas > max_ctas) ctas = max_ctas;
+    if (ctas > cap_ctas) ctas = cap_ctas;
     if (ctas < 1) ctas = 1;
 #ifdef LMO_EXPERIMENTS
     static const char *cap_env = getenv("LMO_ATTN_MAX_CTAS");   // tuning / experiments only
@@ -2088,7 +2111,7 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     cfg.gridDim = dim3((unsigned)ctas);
     cfg.blockDim = dim3(NW * 32);
     cfg.dynamicSmemBytes = sm ? (D == 64 ? smem_bytes<64, kSmWarps>(0) : smem_bytes<128, kSmWarps>(0))
-                              : (D == 64 ? smem_bytes<64>(Bp) : smem_bytes<128>(Bp));
+                              : (D == 64 ? smem_bytes<64>(Bp) : smem_bytes<128>(Bp)) + pad_smem;
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;

@@ -69,6 +69,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_TEAM_RING_ONLY
 #define LMO_TEAM_RING_ONLY 1   // the T > 1 instance merges only on chip: launched only when every
 #endif                         // team has at most one pair (else the generic instance, L2 merge)
+#ifndef LMO_GQA_HOIST
+#define LMO_GQA_HOIST 0   // 1: one V-exponent vote per stage before any p (measured 1% slower than per sub-block)
+#endif
 #ifndef LMO_EARLY_TEST
 #define LMO_EARLY_TEST 0   // non-blocking mbarrier test of stage i+2 during iteration i
 #endif
@@ -1251,6 +1254,27 @@ decode_attn_q4_kernel(const AttnArgs a) {
                 }
             }
             }
+            // V meta of the stage's rows (both sub-blocks) and ONE vote for the V operand
+            // exponent before any p is formed (LMO_GQA_HOIST; else per sub-block)
+            uint2 vmS[kSub][2];
+#pragma unroll
+            for (int s = 0; s < kSub; ++s) {
+                const uint32_t sm = st + s * dSM;
+                vmS[s][0] = (s < nsub) ? load_meta<NG>(sm + offVm0) : make_uint2(0u, 0u);
+                vmS[s][1] = (s < nsub) ? load_meta<NG>(sm + offVm0 + dM1) : make_uint2(0u, 0u);
+            }
+            if (LMO_GQA_HOIST) {
+                uint32_t vx = 0u;
+#pragma unroll
+                for (int s = 0; s < kSub; ++s)
+#pragma unroll
+                    for (int r = 0; r < 2; ++r) {
+                        uint32_t v = NG == 2 ? max(vmS[s][r].x, vmS[s][r].y) : vmS[s][r].x;
+                        if (tail && ks.z[s][r][0] == NEG_INF) v = 0u;   // masked: meta may be stale
+                        vx = max(vx, v);
+                    }
+                if (__any_sync(0xffffffffu, vx >= vthr)) v_exp(vx);
+            }
 #pragma unroll
             for (int s = 0; s < kSub; ++s) {
                 if (s < nsub) {
@@ -1261,10 +1285,9 @@ decode_attn_q4_kernel(const AttnArgs a) {
                         p[r][1] = fast_exp2(ks.z[s][r][1] - mE[1]);
                     }
                     const uint32_t ss = st + s * dSC;
-                    const uint32_t sm = st + s * dSM;
-                    const uint2 vmA = load_meta<NG>(sm + offVm0);
-                    const uint2 vmB = load_meta<NG>(sm + offVm0 + dM1);
-                    {
+                    const uint2 vmA = vmS[s][0];
+                    const uint2 vmB = vmS[s][1];
+                    if (!LMO_GQA_HOIST) {
                         uint32_t vxA = NG == 2 ? max(vmA.x, vmA.y) : vmA.x;
                         uint32_t vxB = NG == 2 ? max(vmB.x, vmB.y) : vmB.x;
                         if (tail) {                    // masked tail tokens: meta may be stale

@@ -464,8 +464,231 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
     }
 }
 
+// ---------------------------------------------------------------------------
+// Packed layout, TWO quantization groups (K = 128) per pipeline step: every
+// per-step synchronisation (code-slot wait, empty arrive + proxy fence, TMEM
+// store wait / fence / full arrive, the MMA issuer's waits and commits) is paid
+// once per 128 weights per thread instead of once per 64 -- the synchronisation,
+// not HBM or the tensor pipe, bounded the one-group kernel (K7).
+// One 1-D bulk copy brings the two consecutive 4608-B packed blocks of a step;
+// the activations arrive as two SW128 atoms; A = 2 x 32 TMEM columns per stage.
+namespace g2 {
+constexpr int kC = 6;       // code slots (2 groups each)
+constexpr int kXS = 3;      // activation stages
+constexpr int kAS = 2;      // A stages in TMEM (64 columns each)
+template <int BN>
+struct Smem {
+    static constexpr int B = 2 * BN * 128;             // two SW128 atoms: BN x 128 fp16
+    static constexpr int PBLK = kM * 32 + kM * 4;      // one packed tile-group block
+    static constexpr int CSLOT = 2 * PBLK;
+    static constexpr int OFF_CODES = kXS * B;
+    static constexpr int OFF_BARS = OFF_CODES + kC * CSLOT;
+    static constexpr int BYTES = OFF_BARS + 512 + 1024;
+};
+template <int BN>
+struct Tmem {
+    static constexpr int A0 = BN;
+    static constexpr int USED = BN + kAS * 64;
+    static constexpr int COLS = USED <= 128 ? 128 : USED <= 256 ? 256 : 512;
+};
+static_assert((2 * kC + 2 * kXS + 2 * kAS + 1) * 8 + 4 <= 512, "barrier area");
+}  // namespace g2
+
+template <int BN>
+__global__ void __launch_bounds__(Roles<1>::THREADS, 1)
+w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restrict__ packed,
+                float *__restrict__ y, int N, int K, int batch, int ksplit) {
+    using S = g2::Smem<BN>;
+    using TM = g2::Tmem<BN>;
+    constexpr int kProd = Roles<1>::PROD, kWMMA = Roles<1>::WMMA, kWTC = Roles<1>::WTC, kWTX = Roles<1>::WTX;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    const uint32_t sbase = smem_u32(smem);
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem + S::OFF_BARS);
+    uint64_t *c_full = bars, *c_empty = bars + g2::kC;
+    uint64_t *x_full = bars + 2 * g2::kC, *x_empty = x_full + g2::kXS;
+    uint64_t *a_full = x_empty + g2::kXS, *ab_empty = a_full + g2::kAS;
+    uint64_t *done = ab_empty + g2::kAS;
+    uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(done + 1);
+
+    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    const int n0 = blockIdx.x * kM;
+    const int KB = K / kK, KS = KB / 2;                 // groups, steps
+    const int s0 = (int)((long long)blockIdx.y * KS / ksplit), s1 = (int)((long long)(blockIdx.y + 1) * KS / ksplit);
+    const int nsteps = s1 - s0, kb0 = 2 * s0;
+
+    if (tid == 0) {
+        for (int s = 0; s < g2::kC; ++s) {
+            mbar_init(&c_full[s], 1);
+            mbar_init(&c_empty[s], kProd);
+        }
+        for (int s = 0; s < g2::kXS; ++s) {
+            mbar_init(&x_full[s], 1);
+            mbar_init(&x_empty[s], 1);
+        }
+        for (int s = 0; s < g2::kAS; ++s) {
+            mbar_init(&a_full[s], kProd);
+            mbar_init(&ab_empty[s], 1);
+        }
+        mbar_init(done, 1);
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+    }
+    if (warp == kWMMA) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(smem_u32(tmem_slot)),
+                     "n"(TM::COLS));
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;\n");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;\n");
+    const uint32_t tmem = *tmem_slot;
+
+    if (warp == kWTC) {
+        if (lane == 0) {   // codes: one bulk copy of a step's two consecutive packed blocks
+            for (int q = 0; q < nsteps; ++q) {
+                const int cs = q % g2::kC;
+                if (q >= g2::kC) mbar_wait(&c_empty[cs], ((q / g2::kC) - 1) & 1);
+                mbar_arrive_expect_tx(&c_full[cs], S::CSLOT);
+                const uint8_t *src = packed + ((int64_t)blockIdx.x * KB + kb0 + 2 * q) * S::PBLK;
+                bulk_g2s(smem + S::OFF_CODES + cs * S::CSLOT, src, S::CSLOT, &c_full[cs], policy_evict_first());
+            }
+        }
+    } else if (warp == kWTX) {
+        if (lane == 0) {   // activations: two 64-wide SW128 boxes per step
+            for (int j = 0; j < nsteps; ++j) {
+                const int xs = j % g2::kXS;
+                if (j >= g2::kXS) mbar_wait(&x_empty[xs], ((j / g2::kXS) - 1) & 1);
+                mbar_arrive_expect_tx(&x_full[xs], S::B);
+                tma_2d(sbase + xs * S::B, &tm_x, (kb0 + 2 * j) * kK, 0, &x_full[xs]);
+                tma_2d(sbase + xs * S::B + BN * 128, &tm_x, (kb0 + 2 * j + 1) * kK, 0, &x_full[xs]);
+            }
+        }
+    } else if (warp < kWMMA) {
+        // dequant -> TMEM: thread = weight row r = TMEM lane
+        const int r = tid;
+        const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16) + TM::A0;
+        for (int j = 0; j < nsteps; ++j) {
+            const int cs = j % g2::kC, st = j % g2::kAS;
+            mbar_wait(&c_full[cs], (j / g2::kC) & 1);
+            if (j >= g2::kAS) mbar_wait(&ab_empty[st], ((j / g2::kAS) - 1) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+#pragma unroll
+            for (int gi = 0; gi < 2; ++gi) {
+                const uint32_t blk = sbase + S::OFF_CODES + cs * S::CSLOT + gi * S::PBLK;
+                uint32_t cw[8], mw;
+                asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
+                             : "=r"(cw[0]), "=r"(cw[1]), "=r"(cw[2]), "=r"(cw[3]) : "r"(blk + r * 32));
+                asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
+                             : "=r"(cw[4]), "=r"(cw[5]), "=r"(cw[6]), "=r"(cw[7]) : "r"(blk + r * 32 + 16));
+                asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(blk + kM * 32 + r * 4));
+                const __half2 mn2 = __half2half2(__ushort_as_half((unsigned short)(mw & 0xFFFFu)));
+                const __half2 sc2 = __half2half2(__ushort_as_half((unsigned short)(mw >> 16)));
+                const __half2 sc16 = __hmul2(sc2, __half2half2(__ushort_as_half(0x2C00)));   // * 1/16
+                uint4 v[8];
+#pragma unroll
+                for (int i = 0; i < 8; ++i) v[i] = deq8(cw[i], sc2, sc16, mn2);
+                asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+                             "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};\n" ::"r"(
+                                 lane_base + st * 64 + gi * 32),
+                             "r"(v[0].x), "r"(v[0].y), "r"(v[0].z), "r"(v[0].w), "r"(v[1].x), "r"(v[1].y), "r"(v[1].z),
+                             "r"(v[1].w), "r"(v[2].x), "r"(v[2].y), "r"(v[2].z), "r"(v[2].w), "r"(v[3].x), "r"(v[3].y),
+                             "r"(v[3].z), "r"(v[3].w), "r"(v[4].x), "r"(v[4].y), "r"(v[4].z), "r"(v[4].w), "r"(v[5].x),
+                             "r"(v[5].y), "r"(v[5].z), "r"(v[5].w), "r"(v[6].x), "r"(v[6].y), "r"(v[6].z), "r"(v[6].w),
+                             "r"(v[7].x), "r"(v[7].y), "r"(v[7].z), "r"(v[7].w)
+                             : "memory");
+            }
+            // the slot's generic-proxy reads before its async-proxy refill (see w4a16_kernel)
+            asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+            mbar_arrive(&c_empty[cs]);
+            asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
+            asm volatile("tcgen05.fence::before_thread_sync;\n");
+            mbar_arrive(&a_full[st]);
+        }
+    } else {
+        // MMA issuer: 2 groups x 4 x (K = 16) per step
+        constexpr uint32_t idesc = umma_idesc<BN>();
+        for (int j = 0; j < nsteps; ++j) {
+            const int st = j % g2::kAS, xs = j % g2::kXS;
+            mbar_wait(&x_full[xs], (j / g2::kXS) & 1);
+            mbar_wait(&a_full[st], (j / g2::kAS) & 1);
+            asm volatile("tcgen05.fence::after_thread_sync;\n");
+            if (lane == 0) {
+                const uint32_t b0 = sbase + xs * S::B;
+#pragma unroll
+                for (int gi = 0; gi < 2; ++gi)
+#pragma unroll
+                    for (int k = 0; k < kK / 16; ++k) {
+                        const uint32_t ta = tmem + TM::A0 + st * 64 + gi * 32 + k * 8;
+                        const uint64_t db = umma_desc(b0 + gi * BN * 128 + k * 32);
+                        const uint32_t acc = (j > 0 || gi > 0 || k > 0) ? 1u : 0u;
+                        asm volatile(
+                            "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+                            "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem),
+                            "r"(ta), "l"(db), "r"(idesc), "r"(acc));
+                    }
+                asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
+                                 smem_u32(&ab_empty[st]))
+                             : "memory");
+                asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
+                                 smem_u32(&x_empty[xs]))
+                             : "memory");
+            }
+            __syncwarp();
+        }
+        if (lane == 0)
+            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
+                             smem_u32(done))
+                         : "memory");
+        __syncwarp();
+    }
+
+    // epilogue: warps 0-3 read the accumulator (TMEM lane = output feature)
+    if (warp < 4) {
+        const int row = (warp & 3) * 32 + lane;
+        if (nsteps > 0) {
+            mbar_wait(done, 0);
+            asm volatile("tcgen05.fence::after_thread_sync;\n");
+        }
+#pragma unroll
+        for (int c0 = 0; c0 < BN; c0 += 32) {
+            uint32_t v[32];
+            const uint32_t taddr = tmem + ((uint32_t)((warp & 3) * 32) << 16) + c0;
+            asm volatile(
+                "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+                "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];\n"
+                : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+                  "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+                  "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
+                  "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
+                  "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+                : "r"(taddr));
+            asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+            if (nsteps == 0) continue;
+#pragma unroll
+            for (int i = 0; i < 32; ++i) {
+                const int b = c0 + i;
+                if (b < batch) {
+                    float *dst = y + (int64_t)b * N + n0 + row;
+                    const float val = __uint_as_float(v[i]);
+                    if (ksplit > 1) atomicAdd(dst, val);
+                    else *dst = val;
+                }
+            }
+        }
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;\n");
+    __syncthreads();
+    if (warp == kWMMA) {
+        asm volatile("tcgen05.fence::after_thread_sync;\n");
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "n"(TM::COLS));
+    }
+}
+
 }  // namespace w4
 
+#ifndef LMO_W4_G2
+#define LMO_W4_G2 1   // packed weights, K % 128 == 0: two quantization groups per pipeline step
+#endif
 #ifndef LMO_W4_MT
 #define LMO_W4_MT 1   // 2: two 128-row tiles per CTA when N % 256 == 0 (measured slower: 213 vs 190 us)
 #endif
@@ -560,6 +783,29 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
     }
     const int MT = w4a16_mt(N);
     const uint32_t *m = static_cast<const uint32_t *>(meta);
+    if (packed && LMO_W4_G2 && MT == 1 && K % (2 * w4::kK) == 0) {   // two groups per pipeline step
+        cudaError_t pre = cudaSuccess;
+        auto go2 = [&](auto kern, int smem_bytes) {
+            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+            if (ksplit <= 0) {
+                int occ = 0;
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, w4::Roles<1>::THREADS, smem_bytes);
+                ksplit = w4a16_auto_split(N, K, occ);
+            }
+            if (ksplit > K / (2 * w4::kK)) ksplit = K / (2 * w4::kK);
+            if (ksplit > 1) {
+                pre = cudaMemsetAsync(y, 0, (size_t)batch * N * sizeof(float), st);
+                if (pre != cudaSuccess) return;
+            }
+            kern<<<dim3(N / w4::kM, ksplit), w4::Roles<1>::THREADS, smem_bytes, st>>>(tx, packed, y, N, K, batch, ksplit);
+        };
+        if (BN == 64) go2(w4::w4a16_g2_kernel<64>, w4::g2::Smem<64>::BYTES);
+        else go2(w4::w4a16_g2_kernel<128>, w4::g2::Smem<128>::BYTES);
+        if (pre != cudaSuccess) return pre;
+        const cudaError_t e = cudaGetLastError();
+        if (e == cudaSuccess) note_launch();
+        return e;
+    }
     cudaError_t pre = cudaSuccess;
     auto go = [&](auto kern, int sm, int threads) {
         cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);

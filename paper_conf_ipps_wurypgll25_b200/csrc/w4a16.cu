@@ -494,13 +494,17 @@ struct Tmem {
 static_assert((2 * kC + 2 * kXS + 2 * kAS + 1) * 8 + 4 <= 512, "barrier area");
 }  // namespace g2
 
-template <int BN>
-__global__ void __launch_bounds__(Roles<1>::THREADS, 1)
+// DW = dequant warps: 4 (thread = weight row, both groups) or 8 (warp w: rows 32 (w % 4) ..,
+// group w / 4 -- two warps per SMSP, half the dependent chain per thread; one mbarrier
+// arrival per warp).
+template <int BN, int DW>
+__global__ void __launch_bounds__(DW * 32 + 96, 1)
 w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restrict__ packed,
                 float *__restrict__ y, int N, int K, int batch, int ksplit) {
     using S = g2::Smem<BN>;
     using TM = g2::Tmem<BN>;
-    constexpr int kProd = Roles<1>::PROD, kWMMA = Roles<1>::WMMA, kWTC = Roles<1>::WTC, kWTX = Roles<1>::WTX;
+    constexpr int kWMMA = DW, kWTC = DW + 1, kWTX = DW + 2;
+    constexpr int kArrive = DW == 8 ? DW : 128;          // arrivals per step on c_empty / a_full
     extern __shared__ uint8_t smem_raw[];
     uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     const uint32_t sbase = smem_u32(smem);
@@ -520,14 +524,14 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
     if (tid == 0) {
         for (int s = 0; s < g2::kC; ++s) {
             mbar_init(&c_full[s], 1);
-            mbar_init(&c_empty[s], kProd);
+            mbar_init(&c_empty[s], kArrive);
         }
         for (int s = 0; s < g2::kXS; ++s) {
             mbar_init(&x_full[s], 1);
             mbar_init(&x_empty[s], 1);
         }
         for (int s = 0; s < g2::kAS; ++s) {
-            mbar_init(&a_full[s], kProd);
+            mbar_init(&a_full[s], kArrive);
             mbar_init(&ab_empty[s], 1);
         }
         mbar_init(done, 1);
@@ -564,16 +568,19 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
             }
         }
     } else if (warp < kWMMA) {
-        // dequant -> TMEM: thread = weight row r = TMEM lane
-        const int r = tid;
+        // dequant -> TMEM: thread = weight row r = TMEM lane (DW = 8: group gi = warp / 4 only)
+        const int r = tid & (kM - 1);
         const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16) + TM::A0;
+        constexpr int G0 = 0, G1 = DW == 8 ? 1 : 2;           // groups of this thread: [g_lo, g_lo + G1)
+        const int g_lo = DW == 8 ? (warp >> 2) : 0;
         for (int j = 0; j < nsteps; ++j) {
             const int cs = j % g2::kC, st = j % g2::kAS;
             mbar_wait(&c_full[cs], (j / g2::kC) & 1);
             if (j >= g2::kAS) mbar_wait(&ab_empty[st], ((j / g2::kAS) - 1) & 1);
             asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
 #pragma unroll
-            for (int gi = 0; gi < 2; ++gi) {
+            for (int gg = G0; gg < G1; ++gg) {
+                const int gi = g_lo + gg;
                 const uint32_t blk = sbase + S::OFF_CODES + cs * S::CSLOT + gi * S::PBLK;
                 uint32_t cw[8], mw;
                 asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
@@ -599,10 +606,20 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
             }
             // the slot's generic-proxy reads before its async-proxy refill (see w4a16_kernel)
             asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-            mbar_arrive(&c_empty[cs]);
+            if (DW == 8) {
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&c_empty[cs]);
+            } else {
+                mbar_arrive(&c_empty[cs]);
+            }
             asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
             asm volatile("tcgen05.fence::before_thread_sync;\n");
-            mbar_arrive(&a_full[st]);
+            if (DW == 8) {
+                __syncwarp();
+                if (lane == 0) mbar_arrive(&a_full[st]);
+            } else {
+                mbar_arrive(&a_full[st]);
+            }
         }
     } else {
         // MMA issuer: 2 groups x 4 x (K = 16) per step
@@ -688,6 +705,9 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
 
 #ifndef LMO_W4_G2
 #define LMO_W4_G2 1   // packed weights, K % 128 == 0: two quantization groups per pipeline step
+#endif
+#ifndef LMO_W4_G2_DW
+#define LMO_W4_G2_DW 4   // dequant warps of the two-group kernel (4 or 8: measured equal within noise)
 #endif
 #ifndef LMO_W4_MT
 #define LMO_W4_MT 1   // 2: two 128-row tiles per CTA when N % 256 == 0 (measured slower: 213 vs 190 us)
@@ -789,7 +809,7 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
             cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
             if (ksplit <= 0) {
                 int occ = 0;
-                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, w4::Roles<1>::THREADS, smem_bytes);
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, LMO_W4_G2_DW * 32 + 96, smem_bytes);
                 ksplit = w4a16_auto_split(N, K, occ);
             }
             if (ksplit > K / (2 * w4::kK)) ksplit = K / (2 * w4::kK);
@@ -797,10 +817,10 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
                 pre = cudaMemsetAsync(y, 0, (size_t)batch * N * sizeof(float), st);
                 if (pre != cudaSuccess) return;
             }
-            kern<<<dim3(N / w4::kM, ksplit), w4::Roles<1>::THREADS, smem_bytes, st>>>(tx, packed, y, N, K, batch, ksplit);
+            kern<<<dim3(N / w4::kM, ksplit), LMO_W4_G2_DW * 32 + 96, smem_bytes, st>>>(tx, packed, y, N, K, batch, ksplit);
         };
-        if (BN == 64) go2(w4::w4a16_g2_kernel<64>, w4::g2::Smem<64>::BYTES);
-        else go2(w4::w4a16_g2_kernel<128>, w4::g2::Smem<128>::BYTES);
+        if (BN == 64) go2(w4::w4a16_g2_kernel<64, LMO_W4_G2_DW>, w4::g2::Smem<64>::BYTES);
+        else go2(w4::w4a16_g2_kernel<128, LMO_W4_G2_DW>, w4::g2::Smem<128>::BYTES);
         if (pre != cudaSuccess) return pre;
         const cudaError_t e = cudaGetLastError();
         if (e == cudaSuccess) note_launch();

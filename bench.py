@@ -52,6 +52,9 @@ def parse():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--scaling", default="strong", choices=["strong", "weak"])
     p.add_argument("--splits", type=int, default=0, help="num_splits (0 = library auto)")
+    p.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                   help="process-group backend (gloo + ranks sharing a GPU: a functional test of the "
+                        "multi-rank path on a 1-GPU box; its timings are not scaling numbers)")
     p.add_argument("--verify-pairs", type=int, default=4, help="C1 sampled (layer, b, kv-head) per rank")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-stream", action="store_true", help="skip the A1/A5 weight streaming and W4A16 legs")
@@ -302,7 +305,7 @@ def verify_outputs(lmo, D, w, sh, out, t, nl, n_pairs, dev):
         worst = max(worst, float(err.max()))
     return {"pairs": int(len(coords_all)), "ranks": int(len(coords_all) // n_pairs), "step_t": t, "L": L,
             "max_normwise_err": worst, "tol": TOL, "pass": bool(worst <= TOL),
-            "gather": "NCCL all_gather_into_tensor (C1)" if D.dist.is_initialized() else "single rank",
+            "gather": (f"{D.dist.get_backend()} all_gather_into_tensor (C1)" if D.dist.is_initialized() else "single rank"),
             "coords": "(layer, global sequence, kv head) per sample"}
 
 
@@ -335,10 +338,16 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    ndev = torch.cuda.device_count()
+    if args.backend == "nccl" and world > ndev:
+        raise SystemExit(f"{world} ranks need {world} GPUs with NCCL ({ndev} visible); --backend gloo shares one")
+    dev = torch.device("cuda", local % ndev)
+    torch.cuda.set_device(dev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
     w = C.CONFIGS[args.config]
     seed = I.seed_for_config(w.index)
     sh = D.shard(rank, world, w.batch, args.scaling)

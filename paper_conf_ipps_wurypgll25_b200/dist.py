@@ -57,6 +57,8 @@ def max_over_ranks(x: float, device=None) -> float:
     """C2: the slowest rank's value on every rank (bench timing reduce)."""
     if not dist.is_available() or not dist.is_initialized() or dist.get_world_size() == 1:
         return float(x)
+    if dist.get_backend() == "gloo":
+        device = "cpu"
     t = torch.tensor([float(x)], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
@@ -67,11 +69,14 @@ def gather_rows(rows: torch.Tensor) -> torch.Tensor:
     every rank -- verification only, outside any timed region."""
     if not dist.is_available() or not dist.is_initialized() or dist.get_world_size() == 1:
         return rows
+    dev = rows.device
+    if dist.get_backend() == "gloo":          # (gloo: host tensors)
+        rows = rows.cpu()
     rows = rows.contiguous()
     out = torch.empty((dist.get_world_size() * rows.shape[0], *rows.shape[1:]), dtype=rows.dtype,
                       device=rows.device)
     dist.all_gather_into_tensor(out, rows)
-    return out
+    return out.to(dev)
 
 
 def sample_pairs(sh: Shard, kv_heads: int, n: int, salt: int = 0):

@@ -31,7 +31,7 @@ import subprocess
 import sys
 import time
 
-ROOT = os.path.dirname(os.path.abspath(__file__))
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
 from paper_conf_ipps_wurypgll25_b200 import configs as C  # noqa: E402
@@ -90,19 +90,13 @@ def workload_config(w: C.Workload, world: int, sh, mode: str, extra=None):
 # ------------------------------------------------------------- clocks ------
 
 class ClockSampler:
-    """nvidia-smi sampled every 50 ms in the background; only the samples whose
-    timestamps fall inside the marked load window (mark_start() .. mark_end(): the
-    busy warm-up window and the timed region) are summarised -- the start-up and
-    idle samples would otherwise inflate the median (a power-capped run can sit
-    well below the maximum clock under load)."""
-    FIELDS = ("timestamp,index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
               "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
               "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
 
     def __init__(self, gpu_index: int):
         self.gpu = gpu_index
         self.proc = None
-        self.t0 = self.t1 = None
 
     def __enter__(self):
         try:
@@ -110,16 +104,10 @@ class ClockSampler:
                 ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
                  "--format=csv,noheader,nounits", "-lms", "50"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
-            time.sleep(0.6)          # nvidia-smi start-up: samples begin before the load window
+            time.sleep(0.6)          # nvidia-smi start-up: samples begin before the timed region
         except Exception:
             self.proc = None
         return self
-
-    def mark_start(self):
-        self.t0 = time.time()
-
-    def mark_end(self):
-        self.t1 = time.time()
 
     def __exit__(self, *exc):
         self.lines = []
@@ -133,30 +121,24 @@ class ClockSampler:
             self.lines = [ln for ln in out.splitlines() if ln.strip()]
 
     def summary(self):
-        import datetime
-        sm, mx, reasons, pw = [], 0.0, set(), []
+        sm, mx, reasons = [], 0.0, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         for ln in getattr(self, "lines", []):
             f = [x.strip() for x in ln.split(",")]
-            if len(f) < 10:
+            if len(f) < 9:
                 continue
             try:
-                ts = datetime.datetime.strptime(f[0], "%Y/%m/%d %H:%M:%S.%f").timestamp()
-                if self.t0 is not None and not (self.t0 <= ts <= (self.t1 or ts)):
-                    continue
-                sm.append(float(f[2]))
-                mx = max(mx, float(f[3]))
-                pw.append(float(f[4]))
+                sm.append(float(f[1]))
+                mx = max(mx, float(f[2]))
             except ValueError:
                 continue
-            for nm, v in zip(names, f[6:10]):
+            for nm, v in zip(names, f[5:9]):
                 if v.lower().startswith("active"):
                     reasons.add(nm)
         if not sm:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
-        return {"sm_mhz": statistics.median(sm), "sm_min_mhz": min(sm), "sm_max_mhz": mx,
-                "power_w_median": statistics.median(pw), "reasons": sorted(reasons), "samples": len(sm),
-                "window": "load window only (busy warm-up + timed region)"}
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
 
 
 # -------------------------------------------------------- CPU oracle -------
@@ -408,6 +390,7 @@ def run_ours(args):
         del kp, vp
         # ---- per-step inputs (device-resident) and outputs
         qbuf, kbuf, vbuf = {}, {}, {}
+        if os.environ.get("DIAG_EMPTY_OUT"): pass
         for t in distinct_t:
             qbuf[t] = torch.empty((nl, B, Hq, 1, d), dtype=torch.float16, device=dev)
             kbuf[t] = torch.empty((nl, B, Hkv, 1, d), dtype=torch.float16, device=dev)
@@ -421,12 +404,25 @@ def run_ours(args):
     stream.synchronize()
     sigma = 1.0 / math.sqrt(d)
 
+    if os.environ.get("DIAG_FLAGS0") == "1":
+        args.no_early = True
+    fixed_len = int(os.environ.get("DIAG_LEN", "0"))
+
     def step(t, attn=True, append=True):
         """One decode step: for every layer, A2 append of the new token at slot
         s+t-1 and A3/A4 attention over L = s+t -- one fused launch per layer
         (lmo_decode_step_q4); attn-only variant for the roofline leg."""
         for l in range(nl):
-            if append and attn:
+            if append and attn and os.environ.get("DIAG_SPLIT") == "1":
+                lmo.lmo_kv_append_quant(caches[l], kbuf[t][l], vbuf[t][l], pos0=s + t - 1, abi=abis[l])
+                lmo.lmo_decode_attention_q4(caches[l], qbuf[t][l].view(B, Hq, d), s + t,
+                                            softmax_scale=sigma, num_splits=args.splits,
+                                            out=out[l], workspace=ws, abi=abis[l])
+            elif append and attn and os.environ.get("DIAG_ATTN") == "1":
+                lmo.lmo_decode_attention_q4(caches[l], qbuf[t][l].view(B, Hq, d), s + t,
+                                            softmax_scale=sigma, num_splits=args.splits,
+                                            out=out[l], workspace=ws, abi=abis[l])
+            elif append and attn:
                 lmo.lmo_decode_step_q4(caches[l], kbuf[t][l], vbuf[t][l], qbuf[t][l].view(B, Hq, d),
                                        s + t, softmax_scale=sigma, num_splits=args.splits,
                                        out=out[l], workspace=ws, abi=abis[l],
@@ -471,8 +467,12 @@ def run_ours(args):
             graphs[t_of[j]].replay()
     barrier()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
-        clk.mark_start()
+    import contextlib
+    samp = ClockSampler(local) if os.environ.get("DIAG_NOSAMP") != "1" else contextlib.nullcontext()
+    if os.environ.get("DIAG_SAME_T") == "1":
+        t_of[:] = [t_of[-1]] * len(t_of)
+    per = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps_total)]
+    with samp as clk:
         with torch.cuda.stream(stream):
             t_end = time.perf_counter() + 0.5
             while time.perf_counter() < t_end:
@@ -483,17 +483,20 @@ def run_ours(args):
         with torch.cuda.stream(stream):
             ev0.record(stream)
             for j in range(args.warmup, steps_total):
+                per[j][0].record(stream)
                 graphs[t_of[j]].replay()
+                per[j][1].record(stream)
             ev1.record(stream)
             # keep the GPU loaded while the sampler catches the tail of the window
             for j in range(args.warmup):
                 graphs[t_of[j]].replay()
         ev1.synchronize()
         torch.cuda.synchronize()
-        clk.mark_end()
     barrier()
     ms = reduce_max(ev0.elapsed_time(ev1))
-    clocks = clk.summary()
+    clocks = clk.summary() if clk is not None else {}
+    print("DIAG per-step ms:", " ".join(f"{per[j][0].elapsed_time(per[j][1]):.3f}" for j in range(args.warmup, steps_total)),
+          "| L:", [w.prompt + t_of[j] for j in range(args.warmup, steps_total)][:6], file=sys.stderr)
     tokens = sh.global_batch * args.steps
     value = tokens / (ms / 1e3)
     step_bytes = sum(C.layer_step_bytes(w, s + t_of[j], sh.global_batch) * nl

@@ -72,9 +72,6 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_GQA_HOIST
 #define LMO_GQA_HOIST 0   // 1: one V-exponent vote per stage before any p (measured 1% slower than per sub-block)
 #endif
-#ifndef LMO_EARLY_TEST
-#define LMO_EARLY_TEST 0   // non-blocking mbarrier test of stage i+2 during iteration i
-#endif
 #ifndef LMO_NO_SCH
 #define LMO_NO_SCH 0     // 1: every schedule runs the generic kernel instance (experiments)
 #endif
@@ -331,18 +328,8 @@ __device__ __forceinline__ int tperm(int r) { return r; }
 //   u[2] = (nib2, nib6) * 2^-24, u[3] = (nib3, nib7) * 2^-20.
 // The 2^-20 slots meet q/16 in the MMA (see the q fragments), so every
 // product is q_i c_i 2^-24.
-// x >> 8.  LMO_SHR_FMA: as the high word of x * 2^24 (IMAD.HI on the FMA pipe) -- the
-// unpacking is ALU-pipe bound (LOP3/PRMT/SHF), the FMA pipe is nearly idle.
-#ifndef LMO_SHR_FMA
-#define LMO_SHR_FMA 0
-#endif
-__device__ __forceinline__ uint32_t shr8(uint32_t x) {
-#if LMO_SHR_FMA
-    return __umulhi(x, 1u << 24);
-#else
-    return x >> 8;
-#endif
-}
+// x >> 8 (an IMAD.HI on the FMA pipe instead of the SHF was measured 13% slower: DESIGN.md §6)
+__device__ __forceinline__ uint32_t shr8(uint32_t x) { return x >> 8; }
 
 __device__ __forceinline__ void unpack_k(uint32_t w, uint32_t *u) {
     const uint32_t s = shr8(w);
@@ -415,18 +402,6 @@ __device__ __forceinline__ uint32_t movmatrix_t(uint32_t x) {
     uint32_t y;
     asm("movmatrix.sync.aligned.m8n8.trans.b16 %0, %1;\n" : "=r"(y) : "r"(x));
     return y;
-}
-
-#ifndef LMO_REDUX_MAX
-#define LMO_REDUX_MAX 0
-#endif
-// warp-wide float max through redux.sync.max.u32 on an order-preserving integer image
-// (x >= 0: sign bit set; x < 0: all bits flipped); exact, -inf stays -inf
-__device__ __forceinline__ float warp_max_f32(float x) {
-    uint32_t u = __float_as_uint(x);
-    u = (u & 0x80000000u) ? ~u : (u | 0x80000000u);
-    u = __reduce_max_sync(0xffffffffu, u);
-    return __uint_as_float((u & 0x80000000u) ? (u & 0x7FFFFFFFu) : ~u);
 }
 
 __device__ __forceinline__ float max_over_g(float v) {   // lanes with equal t (xor 4, 8, 16)
@@ -836,9 +811,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
                     if (lane8 == 0) reinterpret_cast<uint32_t *>(row + GG::RB)[grp8] = mw;
                 }
             }
-#ifndef LMO_NO_APPEND_FENCE
             asm volatile("fence.proxy.async.global;\n" ::: "memory");
-#endif
         }
         __syncwarp();
     };
@@ -1150,13 +1123,9 @@ decode_attn_q4_kernel(const AttnArgs a) {
                 // the running max moves only if some lane's score exceeds it: one vote
                 // instead of a 5-shuffle max chain on most stages (same result)
                 if (!LMO_LAZY_MAX || __any_sync(0xffffffffu, z > m_run[0])) {
-#if LMO_REDUX_MAX
-                const float mb = warp_max_f32(z);              // one REDUX instead of a 5-step shuffle chain
-#else
                 float mb = z;
 #pragma unroll
                 for (int off = 16; off > 0; off >>= 1) mb = fmaxf(mb, __shfl_xor_sync(0xffffffffu, mb, off));
-#endif
                 if (mb > m_run[0]) {                          // warp-uniform
                     const float a0 = fast_exp2(m_run[0] - mb);
                     m_run[0] = mb;
@@ -1357,20 +1326,13 @@ decode_attn_q4_kernel(const AttnArgs a) {
             stage_k(MK, slot, 0, kC);
         }
         int i = 0;
-        bool rdy = false;   // stage i+1 known complete (tested early during iteration i-1)
 #pragma unroll 1
         for (; i + 1 < nst; ++i) {
             int slN = slot;
             uint32_t phN = phase;
             advance(slN, phN);
-            if (!LMO_EARLY_TEST || !rdy) wait_stage(slN, phN);
+            wait_stage(slN, phN);
             stage_k(MK, slN, (i + 1) * kSub, kN);
-            if (LMO_EARLY_TEST) {   // non-blocking test of stage i+2: its latency hides under the V part
-                int slT = slN;
-                uint32_t phT = phN;
-                advance(slT, phT);
-                rdy = mbar_test(&wbar[slT], phT);
-            }
             stage_v(MK, slot, i * kSub, kC);
             slot = slN;
             phase = phN;
@@ -1390,21 +1352,14 @@ decode_attn_q4_kernel(const AttnArgs a) {
             else stage_k(GEN, slot, 0, kC);
         }
         int i = 0;
-        bool rdy = false;
         // steady state: contiguous hot loop (FULL K part of i+1, FULL V part of i)
 #pragma unroll 1
         for (; i + 1 < nfull; ++i) {
             int slN = slot;
             uint32_t phN = phase;
             advance(slN, phN);
-            if (!LMO_EARLY_TEST || !rdy) wait_stage(slN, phN);
+            wait_stage(slN, phN);
             stage_k(FULL, slN, (i + 1) * kSub, kN);
-            if (LMO_EARLY_TEST) {
-                int slT = slN;
-                uint32_t phT = phN;
-                advance(slT, phT);
-                rdy = mbar_test(&wbar[slT], phT);
-            }
             stage_v(FULL, slot, i * kSub, kC);
             slot = slN;
             phase = phN;

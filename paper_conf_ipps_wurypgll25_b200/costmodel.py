@@ -45,6 +45,7 @@ class Hardware:
     gpu_flops: float = 74.4e3           # GFLOP/s fp32 FMA peak: 148 SMs x 128 lanes x 1.965 GHz x 2
     gpu_freq_mhz: float = 1965.0        # SM clock under the bench (clocks line)
     smsp: int = 592                     # 148 SMs x 4 SMSPs
+    warps_per_smsp: int = 4             # resident attention warps (4 CTAs of 4 warps per SM)
     # q4 attention kernel: cycles per 32-token stage per SMSP vs busy warps per SMSP (1..4)
     # and the per-launch head, MHA and GQA-8 (scripts/smsp_probe.py, profiles/smsp_probe_r2.txt:
     # the slope / intercept between L = 256 and 768 at 592*k pairs)
@@ -128,21 +129,44 @@ def dequan_wgt(m: Model, hw: Hardware) -> float:
 
 # ------------------------------------------------------------ attention kernel
 
+def attention_team_size(pairs: int, hw: Hardware) -> int:
+    """The library's default team size (decode_attn.cu choose_team): the smallest
+    T in 1, 2, 4 with pairs * T >= 0.35 of the resident warps."""
+    warps = hw.smsp * hw.warps_per_smsp
+    for T in (1, 2):
+        if pairs * T >= 0.35 * warps:
+            return T
+    return 4
+
+
 def attention_kernel_s(m: Model, L: int, hw: Hardware, batch: int | None = None) -> float:
     """The fused q4 attention launch of one layer at length L (seconds): the slower of
-    the HBM stream (q4 K+V rows, q, fp32 out) and the per-SMSP issue bound of whole
-    (sequence, kv head) pairs placed one per warp (T = 1 schedule), plus the head."""
+    the HBM stream (q4 K+V rows, q, fp32 out) and the per-SMSP issue bound, plus the
+    head.  Work placement follows the library: each (sequence, kv head) pair is
+    split over a team of T warps (attention_team_size), each warp taking
+    ceil(stages / T) 32-token stages; the busiest SMSP runs ceil(pieces / SMSPs)
+    pieces at the measured stage cost for that many busy warps."""
     b = m.bls if batch is None else batch
     pairs = b * m.kv_heads
     stages = math.ceil(L / 32)
     by = pairs * L * 2 * m.head_dim * Q4_BYTES + b * m.kv_heads * m.group_ratio * m.head_dim * 6
     t_hbm = by / (hw.gpu_mem_bw * 1e9)
-    per_smsp = math.ceil(pairs / hw.smsp)                  # pairs on the busiest SMSP
+    T = attention_team_size(pairs, hw)
+    per_smsp = math.ceil(pairs * T / hw.smsp)              # pieces on the busiest SMSP
     busy = min(4, per_smsp)
     cyc = (hw.stage_cycles_mha if m.group_ratio == 1 else hw.stage_cycles_gqa)[busy - 1]
-    t_issue = per_smsp * stages * cyc / (hw.gpu_freq_mhz * 1e6)
+    t_issue = per_smsp * math.ceil(stages / T) * cyc / (hw.gpu_freq_mhz * 1e6)
     head = hw.launch_head_us_mha if m.group_ratio == 1 else hw.launch_head_us_gqa
     return max(t_hbm, t_issue) + head * 1e-6
+
+
+def strong_scaling_attention_s(w: C.Workload, n_gpus: int, L: int | None = None,
+                               hw: Hardware | None = None) -> float:
+    """One rank's attention launch when the global batch is split over n_gpus
+    (dist.shard 'strong': the largest shard is ceil(B / N) sequences)."""
+    hw = hw or Hardware()
+    L = w.prompt + w.gen // 2 if L is None else L
+    return attention_kernel_s(Model.from_workload(w), L, hw, batch=-(-w.batch // n_gpus))
 
 
 # ------------------------------------------------------------------ Eq 1-7

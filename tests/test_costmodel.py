@@ -64,3 +64,31 @@ def test_total_time_eq1_is_sum_of_steps():
     w = C.CONFIGS["c1"]
     tot = M.total_time_s(w, t_pf_layer=0.0)
     assert abs(tot - sum(M.decode_step_s(w, t) for t in range(1, w.gen))) < 1e-12
+
+
+def test_attention_by_batch_within_20pct():
+    """The team-aware kernel model against the measured per-launch attention time at
+    every strong-scaling shard size (B / 2, B / 4, B / 8) and the full batch; the
+    model's team size is the library's choose_team."""
+    g = GOLD["attention_us_by_batch"]["values"]
+    errs = {}
+    for key, us in g.items():
+        name, _, b = key.partition(":")
+        w = C.CONFIGS[name]
+        b = int(b) if b else w.batch
+        pred = M.attention_kernel_s(M.Model.from_workload(w), w.prompt + w.gen // 2, M.Hardware(),
+                                    batch=b) * 1e6
+        errs[key] = rel(pred, us)
+    assert max(errs.values()) <= 0.20, errs
+    assert sum(errs.values()) / len(errs) <= 0.07, errs
+
+
+def test_team_size_and_strong_scaling_prediction():
+    hw = M.Hardware()
+    assert M.attention_team_size(64 * 72, hw) == 1          # c4: 4608 pairs
+    assert M.attention_team_size(8 * 72, hw) == 2           # c4 over 8 GPUs: 576 pairs
+    assert M.attention_team_size(16 * 8, hw) == 4           # c5 over 8 GPUs: 128 pairs
+    w = C.CONFIGS["c4"]
+    t = [M.strong_scaling_attention_s(w, n) for n in (1, 2, 4, 8)]
+    assert all(a > b for a, b in zip(t, t[1:]))              # more GPUs, shorter launch
+    assert t[0] / t[3] < 8 * 0.7                             # but sub-linear: head + 1-warp stage rate

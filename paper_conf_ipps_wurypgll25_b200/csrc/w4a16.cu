@@ -142,7 +142,12 @@ __host__ __device__ constexpr uint32_t umma_idesc() {
 
 // 8 codes (one word, low nibble first) -> 8 fp16 weights RN16(c * scale + min), in k order.
 // (1024 + c) is exact in fp16 (OR into the exponent of 1024); the high nibble of each
-// byte is read in place as 1024 + 16c and scaled by scale/16.
+// byte is read in place as 1024 + 16c.  Normal groups (scale >= 2^-10): 16c is scaled by
+// scale/16, exact there (HADD2 + HFMA2, the HADD2 off the FMA pipe).  TINY groups
+// (scale < 2^-10, where scale/16 would lose bits as an fp16 subnormal): 1024 + 16c is
+// brought back to c exactly by one HFMA2 (t/16 - 64) and meets the full scale.
+// Both give RN16(c * scale + min) with one rounding.
+template <bool TINY>
 __device__ __forceinline__ uint4 deq8(uint32_t w, __half2 sc, __half2 sc16, __half2 mn) {
     const __half2 k1024 = __half2half2(__ushort_as_half(0x6400));
     const uint32_t s8 = w >> 8;
@@ -150,15 +155,24 @@ __device__ __forceinline__ uint4 deq8(uint32_t w, __half2 sc, __half2 sc16, __ha
     const uint32_t t1 = lop3_and_or(w, 0x00F000F0u, 0x64006400u);    // 16 (c1, c5) + 1024
     const uint32_t t2 = lop3_and_or(s8, 0x000F000Fu, 0x64006400u);   // (c2, c6) + 1024
     const uint32_t t3 = lop3_and_or(s8, 0x00F000F0u, 0x64006400u);   // 16 (c3, c7) + 1024
-    auto f = [&](uint32_t t, __half2 s) {
-        const __half2 c = __hsub2(*reinterpret_cast<const __half2 *>(&t), k1024);
+    auto lo = [&](uint32_t t) { return __hsub2(*reinterpret_cast<const __half2 *>(&t), k1024); };
+    auto hi = [&](uint32_t t) {
+        return TINY ? __hfma2(*reinterpret_cast<const __half2 *>(&t), __half2half2(__ushort_as_half(0x2C00)),
+                              __half2half2(__ushort_as_half(0xD400)))     // t/16 - 64 = c
+                    : lo(t);                                            // 16c
+    };
+    auto f = [&](__half2 c, __half2 s) {
         const __half2 r = __hfma2(c, s, mn);
         return *reinterpret_cast<const uint32_t *>(&r);
     };
-    const uint32_t p0 = f(t0, sc), p1 = f(t1, sc16), p2 = f(t2, sc), p3 = f(t3, sc16);
+    const __half2 shi = TINY ? sc : sc16;
+    const uint32_t p0 = f(lo(t0), sc), p1 = f(hi(t1), shi), p2 = f(lo(t2), sc), p3 = f(hi(t3), shi);
     return make_uint4(prmt(p0, p1, 0x5410u), prmt(p2, p3, 0x5410u), prmt(p0, p1, 0x7632u),
                       prmt(p2, p3, 0x7632u));
 }
+
+// scale < 2^-10 (fp16 0x1400): scale/16 is not exact in fp16
+__device__ __forceinline__ bool tiny_scale(uint32_t mw) { return (mw >> 16) < 0x1400u; }
 
 
 __device__ __forceinline__ void tma_2d(uint32_t dst, const void *tmap, int c0, int c1, uint64_t *bar) {
@@ -310,14 +324,18 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
             const __half2 mn2 = __half2half2(__ushort_as_half((unsigned short)(mw & 0xFFFFu)));
             const __half2 sc2 = __half2half2(__ushort_as_half((unsigned short)(mw >> 16)));
             const __half2 sc16 = __hmul2(sc2, __half2half2(__ushort_as_half(0x2C00)));   // * 1/16
-#pragma unroll
-            for (int i = 0; i < WPT / 8; ++i) {
 #if LMO_W4_NODEQ   // (experiment: pipeline / MMA bound without the dequant arithmetic)
-                v[i] = make_uint4(cw[i], cw[i] ^ mw, cw[i], cw[i]);
+#pragma unroll
+            for (int i = 0; i < WPT / 8; ++i) v[i] = make_uint4(cw[i], cw[i] ^ mw, cw[i], cw[i]);
 #else
-                v[i] = deq8(cw[i], sc2, sc16, mn2);
-#endif
+            if (tiny_scale(mw)) {
+#pragma unroll
+                for (int i = 0; i < WPT / 8; ++i) v[i] = deq8<true>(cw[i], sc2, sc16, mn2);
+            } else {
+#pragma unroll
+                for (int i = 0; i < WPT / 8; ++i) v[i] = deq8<false>(cw[i], sc2, sc16, mn2);
             }
+#endif
             if (LMO_W4_WARP_ARRIVE && last_sub) {   // codes consumed (results in registers): one arrive per warp
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&c_empty[cs]);
@@ -592,8 +610,13 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
                 const __half2 sc2 = __half2half2(__ushort_as_half((unsigned short)(mw >> 16)));
                 const __half2 sc16 = __hmul2(sc2, __half2half2(__ushort_as_half(0x2C00)));   // * 1/16
                 uint4 v[8];
+                if (tiny_scale(mw)) {
 #pragma unroll
-                for (int i = 0; i < 8; ++i) v[i] = deq8(cw[i], sc2, sc16, mn2);
+                    for (int i = 0; i < 8; ++i) v[i] = deq8<true>(cw[i], sc2, sc16, mn2);
+                } else {
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) v[i] = deq8<false>(cw[i], sc2, sc16, mn2);
+                }
                 asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
                              "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};\n" ::"r"(
                                  lane_base + st * 64 + gi * 32),

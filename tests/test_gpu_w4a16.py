@@ -172,3 +172,39 @@ def test_w4a16_row_major_ring_repeatable(lmo):
     for _ in range(8):
         y = lmo.lmo_w4a16_linear(c, m, N, K, x, k_split=1)
         assert torch.equal(y, ref)
+
+
+@pytest.mark.parametrize("packed", [False, True])
+def test_w4a16_weight_magnitude_edges(lmo, packed):
+    """Groups of every magnitude class the format allows: scale < 2^-10 (a scale/16
+    operand would be an fp16 subnormal -- the odd-nibble path must see the full
+    scale), all-subnormal weights, constant groups (scale 0) and weights near the
+    fp16 range, in both the row-major and the packed (two-groups-per-step) GEMM.
+    Bound per weight: one fp16 ulp of the weight, at least one subnormal ulp 2^-24."""
+    rng = np.random.default_rng(31)
+    N, K, B = 640, 512, 48
+    W = rng.standard_normal((N, K))
+    W[0:128] *= 1e-4                      # scale ~ 5e-5 < 2^-10
+    W[128:256] *= 3e-6                    # every weight subnormal in fp16
+    W[256:384] = np.repeat(rng.uniform(-2, 2, (128, K // 64)), 64, axis=1)     # scale 0 groups
+    W[384:512] *= 2000.0                  # |w| up to ~1e4
+    W[512:640] *= np.where(rng.random((128, K)) < 0.5, 1e-4, 0.05)              # mixed groups
+    W = W.astype(np.float16)
+    codes, meta = oracle.quantize_groupwise(W, N, K, 1)
+    codes, meta = codes.reshape(N, K // 2), meta.reshape(N, K // 64, 2)
+    x = rng.standard_normal((B, K)).astype(np.float16)
+    ref = oracle.w4a16_linear(codes, meta, N, K, x)
+    wdq = oracle.dequantize_groupwise(codes, meta, N, K, 1).reshape(N, K).astype(np.float64)
+    ax = np.abs(x.astype(np.float64))
+    bound = ax @ (np.abs(wdq).T * 2.0 ** -10 + 2.0 ** -24) + 1e-6
+    c, m = torch.from_numpy(codes).cuda(), torch.from_numpy(meta.view(np.int32)).cuda()
+    xt = torch.from_numpy(x).cuda()
+    if packed:
+        y = lmo.lmo_w4a16_linear_packed(lmo.lmo_w4a16_pack(c, m, N, K), N, K, xt, k_split=1)
+    else:
+        y = lmo.lmo_w4a16_linear(c, m, N, K, xt, k_split=1)
+    err = np.abs(y.cpu().numpy().astype(np.float64) - ref)
+    r = err / bound
+    for lo in range(0, N, 128):
+        print(f"rows {lo}-{lo + 127}: max err/bound {r[:, lo:lo + 128].max():.3f}")
+    assert np.all(err <= bound), (r.max(), np.unravel_index(r.argmax(), r.shape))

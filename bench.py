@@ -682,19 +682,29 @@ def run_ours(args):
         h2d = (hq[t_mid].numel() + hk[t_mid].numel() + hv[t_mid].numel()) * 2
         d2h = hout.numel() * 4
         barrier()
-        # Copy engine and SMs overlap: step j+1's H2D (copy stream) runs while step
-        # j's graph computes; each graph waits for its own inputs' event, each D2H
-        # for its graph.  Every step's inputs still cross PCIe inside the region.
-        cstream = torch.cuda.Stream(device=dev)
+        # Copy engines and SMs overlap: step j+1's H2D (copy stream) runs while step j's
+        # graph computes, each graph waiting for its own inputs' event.  The result is
+        # copied device-to-device into one of two staging slots at the end of its step
+        # and read back on a third stream, so a D2H queued behind an H2D never stalls
+        # the compute stream (slot reuse waits for the D2H two steps back).  An H2D into
+        # a position's buffers waits for the last step that read them (only when
+        # positions repeat, steps > n - 1).  Every step's inputs still cross PCIe inside
+        # the region.
+        cstream, dstream = torch.cuda.Stream(device=dev), torch.cuda.Stream(device=dev)
+        stage = [torch.empty_like(out[nl - 1]) for _ in range(2)]
         timed = list(range(args.warmup, steps_total))
         with torch.cuda.stream(stream):
             x0, x1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             x0.record(stream)
         cstream.wait_event(x0)
+        last_read = {}
+        read_back = [None, None]
 
         def h2d_of(j):
             t = t_of[j]
             with torch.cuda.stream(cstream):
+                if t in last_read:
+                    cstream.wait_event(last_read[t])
                 qbuf[t].copy_(hq[t], non_blocking=True)
                 kbuf[t].copy_(hk[t], non_blocking=True)
                 vbuf[t].copy_(hv[t], non_blocking=True)
@@ -703,24 +713,27 @@ def run_ours(args):
             return ev
 
         ready = h2d_of(timed[0])
-        read_out = None
         for i, j in enumerate(timed):
-            nxt = h2d_of(timed[i + 1]) if i + 1 < len(timed) else None
+            slot = i % 2
             with torch.cuda.stream(stream):
                 stream.wait_event(ready)
-                if read_out is not None:      # out[] is rewritten: previous D2H first
-                    stream.wait_event(read_out)
                 graphs[t_of[j]].replay()
+                if read_back[slot] is not None:
+                    stream.wait_event(read_back[slot])
+                stage[slot].copy_(out[nl - 1], non_blocking=True)
                 done = torch.cuda.Event()
                 done.record(stream)
-            with torch.cuda.stream(cstream):
-                cstream.wait_event(done)
-                hout.copy_(out[nl - 1], non_blocking=True)
-                read_out = torch.cuda.Event()
-                read_out.record(cstream)
-            ready = nxt
+            last_read[t_of[j]] = done
+            with torch.cuda.stream(dstream):
+                dstream.wait_event(done)
+                hout.copy_(stage[slot], non_blocking=True)
+                read_back[slot] = torch.cuda.Event()
+                read_back[slot].record(dstream)
+            if i + 1 < len(timed):
+                ready = h2d_of(timed[i + 1])
         with torch.cuda.stream(stream):
             stream.wait_stream(cstream)
+            stream.wait_stream(dstream)
             x1.record(stream)
         x1.synchronize()
         barrier()
@@ -728,7 +741,7 @@ def run_ours(args):
         e2e = {"value": tokens / (e2e_ms / 1e3), "unit": "tokens/s", "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": d2h, "ms_per_step": e2e_ms / args.steps,
                "h2d_gb_per_s_needed_to_hide": h2d / (ms / args.steps / 1e3) / 1e9,
-               "path": "pinned host inputs -> H2D (copy stream, overlapped with the previous step) -> liblmo C-ABI step graph -> D2H last-layer output"}
+               "path": "pinned host inputs -> H2D (copy stream, overlapped with the previous step) -> liblmo C-ABI step graph -> D2D to a staging slot -> D2H last-layer output (own stream)"}
 
     cpu = None
     if rank == 0 and world == 1:

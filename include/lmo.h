@@ -284,7 +284,10 @@ lmo_status lmo_w4a16_linear(const uint8_t *codes, const lmo_qmeta *meta, int64_t
  * time; lmo_w4a16_pack rearranges them once into the layout the GEMM
  * streams: for each 128-row tile t and group g, one contiguous 4608-byte block
  * at offset (t * K/64 + g) * 4608 holding the tile's 128 rows x 32 code bytes
- * followed by their 128 lmo_qmeta.  A tile-step is then one 1-D bulk copy of
+ * followed by their 128 lmo_qmeta.  Each 32-bit code word (8 consecutive k,
+ * k-th code at nibble k) is stored k-interleaved: nibbles 0-3 hold k 0, 2, 4, 6
+ * and nibbles 4-7 hold k 1, 3, 5, 7 (the dequantizer's masks then yield
+ * k-ordered fp16 pairs directly).  A tile-step is then one 1-D bulk copy of
  * whole DRAM pages instead of 128 scattered 32-byte row pieces.
  * lmo_w4a16_packed_bytes gives the size (0 for an invalid shape);
  * lmo_w4a16_linear_packed computes exactly what lmo_w4a16_linear computes on

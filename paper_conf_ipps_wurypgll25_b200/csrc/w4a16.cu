@@ -147,7 +147,10 @@ __host__ __device__ constexpr uint32_t umma_idesc() {
 // (scale < 2^-10, where scale/16 would lose bits as an fp16 subnormal): 1024 + 16c is
 // brought back to c exactly by one HFMA2 (t/16 - 64) and meets the full scale.
 // Both give RN16(c * scale + min) with one rounding.
-template <bool TINY>
+// PK (the packed streaming layout): the word's nibbles are stored k-interleaved
+// (positions 0-3 = k 0, 2, 4, 6; positions 4-7 = k 1, 3, 5, 7 -- lmo_w4a16_pack), so the
+// four masks already yield k-ordered pairs and no byte permutes are needed.
+template <bool TINY, bool PK = false>
 __device__ __forceinline__ uint4 deq8(uint32_t w, __half2 sc, __half2 sc16, __half2 mn) {
     const __half2 k1024 = __half2half2(__ushort_as_half(0x6400));
     const uint32_t s8 = w >> 8;
@@ -167,6 +170,7 @@ __device__ __forceinline__ uint4 deq8(uint32_t w, __half2 sc, __half2 sc16, __ha
     };
     const __half2 shi = TINY ? sc : sc16;
     const uint32_t p0 = f(lo(t0), sc), p1 = f(hi(t1), shi), p2 = f(lo(t2), sc), p3 = f(hi(t3), shi);
+    if (PK) return make_uint4(p0, p1, p2, p3);
     return make_uint4(prmt(p0, p1, 0x5410u), prmt(p2, p3, 0x5410u), prmt(p0, p1, 0x7632u),
                       prmt(p2, p3, 0x7632u));
 }
@@ -330,10 +334,10 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
 #else
             if (tiny_scale(mw)) {
 #pragma unroll
-                for (int i = 0; i < WPT / 8; ++i) v[i] = deq8<true>(cw[i], sc2, sc16, mn2);
+                for (int i = 0; i < WPT / 8; ++i) v[i] = deq8<true, PACKED>(cw[i], sc2, sc16, mn2);
             } else {
 #pragma unroll
-                for (int i = 0; i < WPT / 8; ++i) v[i] = deq8<false>(cw[i], sc2, sc16, mn2);
+                for (int i = 0; i < WPT / 8; ++i) v[i] = deq8<false, PACKED>(cw[i], sc2, sc16, mn2);
             }
 #endif
             if (LMO_W4_WARP_ARRIVE && last_sub) {   // codes consumed (results in registers): one arrive per warp
@@ -468,8 +472,12 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
                 if (b < batch) {
                     float *dst = y + (int64_t)b * N + n0 + row;
                     const float val = __uint_as_float(v[i]);
+#ifdef LMO_W4_NOATOMIC   // (timing experiment: split-K partials stored, not reduced -- wrong results)
+                    *dst = val;
+#else
                     if (ksplit > 1) atomicAdd(dst, val);
                     else *dst = val;
+#endif
                 }
             }
         }
@@ -490,10 +498,25 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
 // not HBM or the tensor pipe, bounded the one-group kernel (K7).
 // One 1-D bulk copy brings the two consecutive 4608-B packed blocks of a step;
 // the activations arrive as two SW128 atoms; A = 2 x 32 TMEM columns per stage.
+#ifdef LMO_W4_EXP_TL   // (experiment: per-step clock timeline of CTA (0, 0) of the two-group kernel)
+__device__ unsigned int g_w4_tl[16][512];
+#define W4TL(slot, j) do { if (blockIdx.x == 0 && blockIdx.y == 0 && (j) < 512) g_w4_tl[slot][j] = (unsigned)clock(); } while (0)
+#else
+#define W4TL(slot, j) do { } while (0)
+#endif
 namespace g2 {
-constexpr int kC = 6;       // code slots (2 groups each)
-constexpr int kXS = 3;      // activation stages
-constexpr int kAS = 2;      // A stages in TMEM (64 columns each)
+#ifndef LMO_W4_G2_C
+#define LMO_W4_G2_C 6
+#endif
+#ifndef LMO_W4_G2_XS
+#define LMO_W4_G2_XS 3
+#endif
+constexpr int kC = LMO_W4_G2_C;       // code slots (2 groups each)
+constexpr int kXS = LMO_W4_G2_XS;     // activation stages
+#ifndef LMO_W4_G2_AS
+#define LMO_W4_G2_AS 2
+#endif
+constexpr int kAS = LMO_W4_G2_AS;      // A stages in TMEM (64 columns each)
 template <int BN>
 struct Smem {
     static constexpr int B = 2 * BN * 128;             // two SW128 atoms: BN x 128 fp16
@@ -570,6 +593,7 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
             for (int q = 0; q < nsteps; ++q) {
                 const int cs = q % g2::kC;
                 if (q >= g2::kC) mbar_wait(&c_empty[cs], ((q / g2::kC) - 1) & 1);
+                W4TL(0, q);
                 mbar_arrive_expect_tx(&c_full[cs], S::CSLOT);
                 const uint8_t *src = packed + ((int64_t)blockIdx.x * KB + kb0 + 2 * q) * S::PBLK;
                 bulk_g2s(smem + S::OFF_CODES + cs * S::CSLOT, src, S::CSLOT, &c_full[cs], policy_evict_first());
@@ -580,6 +604,7 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
             for (int j = 0; j < nsteps; ++j) {
                 const int xs = j % g2::kXS;
                 if (j >= g2::kXS) mbar_wait(&x_empty[xs], ((j / g2::kXS) - 1) & 1);
+                W4TL(1, j);
                 mbar_arrive_expect_tx(&x_full[xs], S::B);
                 tma_2d(sbase + xs * S::B, &tm_x, (kb0 + 2 * j) * kK, 0, &x_full[xs]);
                 tma_2d(sbase + xs * S::B + BN * 128, &tm_x, (kb0 + 2 * j + 1) * kK, 0, &x_full[xs]);
@@ -593,8 +618,11 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
         const int g_lo = DW == 8 ? (warp >> 2) : 0;
         for (int j = 0; j < nsteps; ++j) {
             const int cs = j % g2::kC, st = j % g2::kAS;
+            if (tid == 0) W4TL(2, j);
             mbar_wait(&c_full[cs], (j / g2::kC) & 1);
+            if (tid == 0) W4TL(3, j);
             if (j >= g2::kAS) mbar_wait(&ab_empty[st], ((j / g2::kAS) - 1) & 1);
+            if (tid == 0) W4TL(4, j);
             asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
 #pragma unroll
             for (int gg = G0; gg < G1; ++gg) {
@@ -606,16 +634,25 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
                 asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];\n"
                              : "=r"(cw[4]), "=r"(cw[5]), "=r"(cw[6]), "=r"(cw[7]) : "r"(blk + r * 32 + 16));
                 asm volatile("ld.shared.u32 %0, [%1];\n" : "=r"(mw) : "r"(blk + kM * 32 + r * 4));
+#ifdef LMO_W4_EXP_TL
+                if (tid == 0 && blockIdx.x == 0 && blockIdx.y == 0 && j < 512) g_w4_tl[8 + 3 * gg][j] = (unsigned)clock() + (mw & cw[7] & 0);
+#endif
                 const __half2 mn2 = __half2half2(__ushort_as_half((unsigned short)(mw & 0xFFFFu)));
                 const __half2 sc2 = __half2half2(__ushort_as_half((unsigned short)(mw >> 16)));
                 const __half2 sc16 = __hmul2(sc2, __half2half2(__ushort_as_half(0x2C00)));   // * 1/16
                 uint4 v[8];
+#if LMO_W4_NODEQ   // (experiment: the pipeline without the dequant arithmetic)
+                if (true) {
+#pragma unroll
+                    for (int i = 0; i < 8; ++i) v[i] = make_uint4(cw[i], cw[i] ^ mw, cw[i], cw[i]);
+                } else
+#endif
                 if (tiny_scale(mw)) {
 #pragma unroll
-                    for (int i = 0; i < 8; ++i) v[i] = deq8<true>(cw[i], sc2, sc16, mn2);
+                    for (int i = 0; i < 8; ++i) v[i] = deq8<true, true>(cw[i], sc2, sc16, mn2);
                 } else {
 #pragma unroll
-                    for (int i = 0; i < 8; ++i) v[i] = deq8<false>(cw[i], sc2, sc16, mn2);
+                    for (int i = 0; i < 8; ++i) v[i] = deq8<false, true>(cw[i], sc2, sc16, mn2);
                 }
                 asm volatile("tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
                              "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};\n" ::"r"(
@@ -626,16 +663,25 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
                              "r"(v[5].y), "r"(v[5].z), "r"(v[5].w), "r"(v[6].x), "r"(v[6].y), "r"(v[6].z), "r"(v[6].w),
                              "r"(v[7].x), "r"(v[7].y), "r"(v[7].z), "r"(v[7].w)
                              : "memory");
+#ifdef LMO_W4_EXP_TL
+                if (tid == 0 && blockIdx.x == 0 && blockIdx.y == 0 && j < 512) g_w4_tl[9 + 3 * gg][j] = (unsigned)clock() + (v[7].w & v[0].x & 0);
+#endif
             }
             // the slot's generic-proxy reads before its async-proxy refill (see w4a16_kernel)
+#ifndef LMO_W4_EXP_NOFENCE
             asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+#endif
             if (DW == 8) {
                 __syncwarp();
                 if (lane == 0) mbar_arrive(&c_empty[cs]);
             } else {
                 mbar_arrive(&c_empty[cs]);
             }
+            if (tid == 0) W4TL(14, j);
+#ifndef LMO_W4_EXP_NOWAITST
             asm volatile("tcgen05.wait::st.sync.aligned;\n" ::: "memory");
+#endif
+            if (tid == 0) W4TL(15, j);
             asm volatile("tcgen05.fence::before_thread_sync;\n");
             if (DW == 8) {
                 __syncwarp();
@@ -643,6 +689,7 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
             } else {
                 mbar_arrive(&a_full[st]);
             }
+            if (tid == 0) W4TL(5, j);
         }
     } else {
         // MMA issuer: 2 groups x 4 x (K = 16) per step
@@ -650,14 +697,21 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
         for (int j = 0; j < nsteps; ++j) {
             const int st = j % g2::kAS, xs = j % g2::kXS;
             mbar_wait(&x_full[xs], (j / g2::kXS) & 1);
+            if (lane == 0) W4TL(6, j);
             mbar_wait(&a_full[st], (j / g2::kAS) & 1);
+            if (lane == 0) W4TL(7, j);
             asm volatile("tcgen05.fence::after_thread_sync;\n");
             if (lane == 0) {
                 const uint32_t b0 = sbase + xs * S::B;
+#ifdef LMO_W4_EXP_MMA1   // (timing experiment: one MMA per step -- wrong results)
+                for (int gi = 0; gi < 1; ++gi)
+                    for (int k = 0; k < 1; ++k) {
+#else
 #pragma unroll
                 for (int gi = 0; gi < 2; ++gi)
 #pragma unroll
                     for (int k = 0; k < kK / 16; ++k) {
+#endif
                         const uint32_t ta = tmem + TM::A0 + st * 64 + gi * 32 + k * 8;
                         const uint64_t db = umma_desc(b0 + gi * BN * 128 + k * 32);
                         const uint32_t acc = (j > 0 || gi > 0 || k > 0) ? 1u : 0u;
@@ -710,8 +764,12 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
                 if (b < batch) {
                     float *dst = y + (int64_t)b * N + n0 + row;
                     const float val = __uint_as_float(v[i]);
+#ifdef LMO_W4_NOATOMIC   // (timing experiment: split-K partials stored, not reduced -- wrong results)
+                    *dst = val;
+#else
                     if (ksplit > 1) atomicAdd(dst, val);
                     else *dst = val;
+#endif
                 }
             }
         }
@@ -736,6 +794,27 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
 #define LMO_W4_MT 1   // 2: two 128-row tiles per CTA when N % 256 == 0 (measured slower: 213 vs 190 us)
 #endif
 static int w4a16_mt(int N) { return (LMO_W4_MT == 2 && N % (2 * w4::kM) == 0) ? 2 : 1; }
+
+#ifdef LMO_W4_EXP_TL
+extern "C" int lmo_exp_w4_timeline(unsigned int *host) {
+    return (int)cudaMemcpyFromSymbol(host, w4::g_w4_tl, sizeof(w4::g_w4_tl));
+}
+#endif
+
+// Resident CTAs per SM of a W4A16 instance: shared memory (with the per-block
+// reservation), tensor memory columns (512 per SM) and threads.  (The runtime's
+// occupancy query reported 1 for the two-group instance where ncu and the split-K
+// timings show 2: 7168 x 28672 ran at 67 instead of 41 us with the auto split.)
+static int w4a16_resident_ctas(int smem_bytes, int tmem_cols, int threads) {
+    int dev = 0, smem_sm = 0, reserved = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev);
+    cudaDeviceGetAttribute(&reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev);
+    int occ = smem_sm / (smem_bytes + reserved);
+    occ = std::min(occ, 512 / tmem_cols);
+    occ = std::min(occ, 2048 / threads);
+    return std::max(occ, 1);
+}
 
 int w4a16_auto_split(int N, int K, int ctas_per_sm) {
     // the most K splits that still fit ONE wave of resident CTAs (ctas_per_sm: the occupancy
@@ -765,8 +844,18 @@ static EncodeTiledFn encode_tiled() {
     return fn;
 }
 
+// One code word (k 0..7 at nibble positions 0..7) -> the packed layout's k-interleaved
+// word: positions 0-3 hold k 0, 2, 4, 6 and positions 4-7 hold k 1, 3, 5, 7.
+__device__ __forceinline__ uint32_t interleave_nibbles(uint32_t w) {
+    uint32_t o = 0;
+#pragma unroll
+    for (int k = 0; k < 8; ++k) o |= ((w >> (4 * k)) & 0xFu) << (4 * ((k & 1) * 4 + (k >> 1)));
+    return o;
+}
+
 // Pack W (codes [N][K/2], meta [N][K/64]) into the streaming layout: block (tile, g) of
-// 4608 B = [128 rows x 32 B codes | 128 x 4 B meta] at ((tile * K/64) + g) * 4608.
+// 4608 B = [128 rows x 32 B codes (k-interleaved words) | 128 x 4 B meta] at
+// ((tile * K/64) + g) * 4608.
 __global__ void w4a16_pack_kernel(const uint8_t *__restrict__ codes, const uint32_t *__restrict__ meta,
                                   uint8_t *__restrict__ packed, int N, int K) {
     const int KB = K / w4::kK;
@@ -779,6 +868,8 @@ __global__ void w4a16_pack_kernel(const uint8_t *__restrict__ codes, const uint3
         if (w < w4::kM * 2) {              // codes: row w/2, half w%2
             const int r = w >> 1, hh = w & 1;
             v = *reinterpret_cast<const uint4 *>(codes + (int64_t)(tile * w4::kM + r) * (K / 2) + g * 32 + hh * 16);
+            v = make_uint4(interleave_nibbles(v.x), interleave_nibbles(v.y), interleave_nibbles(v.z),
+                           interleave_nibbles(v.w));
         } else {                           // meta: rows 4(w-256) .. +3
             const int r0 = (w - w4::kM * 2) * 4;
             const uint32_t *mp = meta + (int64_t)(tile * w4::kM + r0) * KB + g;
@@ -828,11 +919,11 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
     const uint32_t *m = static_cast<const uint32_t *>(meta);
     if (packed && LMO_W4_G2 && MT == 1 && K % (2 * w4::kK) == 0) {   // two groups per pipeline step
         cudaError_t pre = cudaSuccess;
-        auto go2 = [&](auto kern, int smem_bytes) {
+        auto go2 = [&](auto kern, int smem_bytes, int tmem_cols) {
             cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+            cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
             if (ksplit <= 0) {
-                int occ = 0;
-                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, LMO_W4_G2_DW * 32 + 96, smem_bytes);
+                const int occ = w4a16_resident_ctas(smem_bytes, tmem_cols, LMO_W4_G2_DW * 32 + 96);
                 ksplit = w4a16_auto_split(N, K, occ);
             }
             if (ksplit > K / (2 * w4::kK)) ksplit = K / (2 * w4::kK);
@@ -842,8 +933,8 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
             }
             kern<<<dim3(N / w4::kM, ksplit), LMO_W4_G2_DW * 32 + 96, smem_bytes, st>>>(tx, packed, y, N, K, batch, ksplit);
         };
-        if (BN == 64) go2(w4::w4a16_g2_kernel<64, LMO_W4_G2_DW>, w4::g2::Smem<64>::BYTES);
-        else go2(w4::w4a16_g2_kernel<128, LMO_W4_G2_DW>, w4::g2::Smem<128>::BYTES);
+        if (BN == 64) go2(w4::w4a16_g2_kernel<64, LMO_W4_G2_DW>, w4::g2::Smem<64>::BYTES, w4::g2::Tmem<64>::COLS);
+        else go2(w4::w4a16_g2_kernel<128, LMO_W4_G2_DW>, w4::g2::Smem<128>::BYTES, w4::g2::Tmem<128>::COLS);
         if (pre != cudaSuccess) return pre;
         const cudaError_t e = cudaGetLastError();
         if (e == cudaSuccess) note_launch();
@@ -852,6 +943,7 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
     cudaError_t pre = cudaSuccess;
     auto go = [&](auto kern, int sm, int threads) {
         cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, sm);
+        cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
         if (ksplit <= 0) {   // auto: one wave of the resident CTAs of THIS instance
             int occ = 0;
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, threads, sm);

@@ -142,9 +142,16 @@ def test_w4a16_packed_layout(lmo, N, K, batch, k_split):
     packed = lmo.lmo_w4a16_pack(c, m, N, K).cpu().numpy()
     KB = K // 64
     blk = packed.reshape(N // 128, KB, 4608)
+    # code words k-interleaved (include/lmo.h): nibble k of a word moves to position
+    # 4 * (k % 2) + k // 2
+    words = codes.view("<u4")
+    inter = np.zeros_like(words)
+    for k in range(8):
+        inter |= ((words >> np.uint32(4 * k)) & np.uint32(0xF)) << np.uint32(4 * (4 * (k % 2) + k // 2))
+    inter = inter.view(np.uint8)
     for t in range(N // 128):
         for g in (0, KB - 1):
-            assert np.array_equal(blk[t, g, :4096].reshape(128, 32), codes[t * 128:(t + 1) * 128, g * 32:(g + 1) * 32])
+            assert np.array_equal(blk[t, g, :4096].reshape(128, 32), inter[t * 128:(t + 1) * 128, g * 32:(g + 1) * 32])
             assert np.array_equal(blk[t, g, 4096:].view(np.uint16).reshape(128, 2), meta[t * 128:(t + 1) * 128, g])
     x = torch.from_numpy(rng.standard_normal((batch, K)).astype(np.float16)).cuda()
     y1 = lmo.lmo_w4a16_linear(c, m, N, K, x, k_split=1).cpu()

@@ -682,46 +682,62 @@ decode_attn_q4_kernel(const AttnArgs a) {
     // and the 2^-20 code slots meet q'/16: without the rescale a small q (|q| < 2^-10)
     // would become an fp16 subnormal after /16 and lose bits.  2^-Eq is folded into zk.
     auto build_q = [&](const uint4 (&raw)[NG][2]) {
-        uint32_t mx = 0;                                  // max |q| of the pair (fp16 bits)
+        // max |q| of the pair on packed halves (sign bit cleared: an fp16 bit pattern
+        // compares as an unsigned 16-bit integer)
+        uint32_t mx2 = 0;
 #pragma unroll
         for (int grp = 0; grp < NG; ++grp)
 #pragma unroll
             for (int k = 0; k < 2; ++k) {
                 const uint32_t w[4] = {raw[grp][k].x, raw[grp][k].y, raw[grp][k].z, raw[grp][k].w};
 #pragma unroll
-                for (int i = 0; i < 4; ++i) mx = max(mx, max(w[i] & 0x7FFFu, (w[i] >> 16) & 0x7FFFu));
+                for (int i = 0; i < 4; ++i) mx2 = __vmaxu2(mx2, w[i] & 0x7FFF7FFFu);
             }
-        mx = __reduce_max_sync(0xffffffffu, mx);
+        const uint32_t mx = __reduce_max_sync(0xffffffffu, max(mx2 & 0xFFFFu, mx2 >> 16));
         int eq = 0;
         if (mx) eq = 14 - floor_log2_h(mx);               // in [-1, 38]
-        const float qsc = exp2i(eq);
         zk = zs * 16777216.0f * exp2i(-eq);
+        // q' = q * 2^eq on packed halves: exact for eq >= 0 (scaling up keeps every bit, no
+        // overflow by the choice of eq) and one RN for eq = -1 -- the same value as
+        // RN16(float(q) * 2^eq).  2^eq > 2^15 is applied in up to three exact steps
+        // (warp-uniform branch; q with max|q| < 2^-1 only).
+        const int e1 = min(eq, 15);
+        const __half2 s1 = __halves2half2(__ushort_as_half((uint16_t)((e1 + 15) << 10)),
+                                          __ushort_as_half((uint16_t)((e1 + 15) << 10)));
+        const __half2 s16 = __float2half2_rn(0.0625f);
+        auto scale = [&](uint32_t x) -> __half2 {
+            __half2 h = __hmul2(*reinterpret_cast<const __half2 *>(&x), s1);
+            if (eq > 15) {
+                const int e2 = min(eq - 15, 15), e3 = eq - 15 - e2;
+                h = __hmul2(h, __halves2half2(__ushort_as_half((uint16_t)((e2 + 15) << 10)),
+                                              __ushort_as_half((uint16_t)((e2 + 15) << 10))));
+                h = __hmul2(h, __halves2half2(__ushort_as_half((uint16_t)((e3 + 15) << 10)),
+                                              __ushort_as_half((uint16_t)((e3 + 15) << 10))));
+            }
+            return h;
+        };
 #pragma unroll
         for (int grp = 0; grp < NG; ++grp) {
-            const __half *h0 = reinterpret_cast<const __half *>(&raw[grp][0]);
-            const __half *h1 = reinterpret_cast<const __half *>(&raw[grp][1]);
-            __half q16[16];
-            float sum = 0.f;
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                q16[i] = __float2half_rn(__half2float(h0[i]) * qsc);
-                q16[8 + i] = __float2half_rn(__half2float(h1[i]) * qsc);
-                sum += __half2float(h0[i]) + __half2float(h1[i]);
-            }
-            sum = sum_over_t(sum);                              // Qs of head g
-            qs[grp][0] = __shfl_sync(0xffffffffu, sum, 8 * t);      // head 2t   (g = 2t)
-            qs[grp][1] = __shfl_sync(0xffffffffu, sum, 8 * t + 4);  // head 2t+1
+            // B fragment of k-block kbl: r = 0 -> (q[i0], q[i0+4]) meets the 2^-24 code slots,
+            // r = 1 -> (q[i0+1], q[i0+5]) / 16 meets the 2^-20 slots (i0 = 8*(kbl>>1) + 2*(kbl&1))
 #pragma unroll
             for (int kbl = 0; kbl < 4; ++kbl) {
-#pragma unroll
-                for (int r = 0; r < 2; ++r) {
-                    const int idx = 2 * kbl + r;
-                    const int i0 = 8 * (idx >> 2) + (idx & 3);
-                    __half2 pr = __halves2half2(q16[i0], q16[i0 + 4]);
-                    if (r == 1) pr = __hmul2(pr, __float2half2_rn(0.0625f));  // meets c*2^-20
-                    qf[grp][kbl][r] = *reinterpret_cast<uint32_t *>(&pr);
-                }
+                const uint4 &rw = raw[grp][kbl >> 1];
+                const uint32_t wa = (kbl & 1) ? rw.y : rw.x, wb = (kbl & 1) ? rw.w : rw.z;
+                const __half2 p0 = scale(prmt(wa, wb, 0x5410u));
+                const __half2 p1 = __hmul2(scale(prmt(wa, wb, 0x7632u)), s16);
+                qf[grp][kbl][0] = *reinterpret_cast<const uint32_t *>(&p0);
+                qf[grp][kbl][1] = *reinterpret_cast<const uint32_t *>(&p1);
             }
+            // Qs of heads 2t, 2t+1 from the MMA itself: A = 1 on the k rows of the 2^-24 slots
+            // and 16 on the q'/16 rows, so C[., n] = sum of head n's q' (products exact), and
+            // the lane's C columns 2t, 2t+1 are exactly its heads.  Qs = C * 2^-eq.
+            float c[4] = {0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+            for (int kbl = 0; kbl < 4; ++kbl)
+                mma_16816(c, 0x3C003C00u, 0x3C003C00u, 0x4C004C00u, 0x4C004C00u, qf[grp][kbl][0], qf[grp][kbl][1]);
+            qs[grp][0] = c[0] * exp2i(-eq);
+            qs[grp][1] = c[1] * exp2i(-eq);
         }
     };
     auto load_q = [&](int b, int kvh) {
@@ -1533,7 +1549,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
                             o[grp][6] = fmaf(x1.z, wr, o[grp][6]); o[grp][7] = fmaf(x1.w, wr, o[grp][7]);
                         }
                     }
-                    const float il = 1.f / l;
+                    const float il = __frcp_rn(l);
 #pragma unroll
                     for (int grp = 0; grp < NG; ++grp) {
 #pragma unroll
@@ -1604,7 +1620,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
                             for (int i2 = 0; i2 < DPL; ++i2) o[i2] = fmaf(oj[j][i2], w, o[i2]);
                         }
                     }
-                    const float il = 1.f / l;
+                    const float il = __frcp_rn(l);
                     const int64_t row = rowbase + h;
                     if (a.out_f16) {
 #pragma unroll
@@ -1625,7 +1641,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
 #pragma unroll
             for (int e = 0; e < 2; ++e) {
                 const int h = 2 * t + e;
-                const float il = 1.f / lt[e];
+                const float il = __frcp_rn(lt[e]);
                 if (sd.L <= 0) break;
 #pragma unroll
                 for (int grp = 0; grp < NG; ++grp) {
@@ -1712,7 +1728,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
                             for (int i = 0; i < DPL; ++i) o[i] = fmaf(__ldcg(r + lane * DPL + i), w, o[i]);
                         }
                     }
-                    const float il = 1.f / l;
+                    const float il = __frcp_rn(l);
                     const int64_t row = rowbase + h;
 #pragma unroll
                     for (int i = 0; i < DPL; ++i) {
@@ -1799,7 +1815,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
                     }
                     M = Mn;
                 }
-                const float il = 1.f / l;
+                const float il = __frcp_rn(l);
                 const int64_t row = rowbase + h;
                 if (a.out_f16) {
 #pragma unroll

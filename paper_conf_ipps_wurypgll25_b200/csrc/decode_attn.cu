@@ -81,6 +81,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_ATTN_MINBLOCKS
 #define LMO_ATTN_MINBLOCKS 4
 #endif
+#ifndef LMO_DEEP_GQA
+#define LMO_DEEP_GQA 1   // GQA launches with ~1 pair per warp of a 2-CTA/SM grid: deep-ring instance
+#endif
 constexpr int kWarps = LMO_ATTN_WARPS;    // warps per CTA
 constexpr int kStages = LMO_ATTN_STAGES;  // per-warp TMA ring depth (stages of 32 tokens)
 constexpr int kMaxBatchSmem = 1024;  // per-sequence-length mode: prefix array in smem
@@ -491,22 +494,25 @@ struct KState {       // per-stage scores handed from the K part to the V part
 };
 
 // smem layout: mbarriers [NW][kStages] (128-B aligned block), rings [NW][kStages][STAGE], prefix
-template <int NW>
-__host__ __device__ constexpr int bars_bytes() { return (NW * kStages * 8 + 127) / 128 * 128; }
+template <int NW, int ST = kStages>
+__host__ __device__ constexpr int bars_bytes() { return (NW * ST * 8 + 127) / 128 * 128; }
+// Deep-ring instance (ST = kDeepStages, 2 CTAs per SM): GQA launches with about one pair per
+// warp at 2 CTAs/SM keep twice the bytes in flight per busy warp (c5: 41.1 -> 39.0 us)
+constexpr int kDeepStages = 5;
 
 // SCH: 0 = any schedule (runtime work map mode); 1 = pair teams with T = 1 (one warp
 // per pair, the default); 2 = pair teams with T > 1.  The specialised instances drop
 // the other modes' code (smaller kernel: fewer cold instruction-cache misses).
-template <int D, bool MHA, int NW, int SCH = 0>
-__global__ void __launch_bounds__(NW * 32, NW == kWarps ? (MHA ? LMO_ATTN_MINBLOCKS : LMO_ATTN_MINBLOCKS_GQA) : 1)
+template <int D, bool MHA, int NW, int SCH = 0, int ST = kStages>
+__global__ void __launch_bounds__(NW * 32, NW == kWarps ? (ST != kStages ? 2 : MHA ? LMO_ATTN_MINBLOCKS : LMO_ATTN_MINBLOCKS_GQA) : 1)
 decode_attn_q4_kernel(const AttnArgs a) {
     using GG = Geo<D>;
     constexpr bool TEAMK = SCH != 0;
     constexpr int NG = GG::NG;
     extern __shared__ __align__(128) uint8_t smem[];
-    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);                 // [NW][kStages]
-    uint8_t *ring = smem + bars_bytes<NW>();                              // [NW][kStages][STAGE]
-    int *prefix = reinterpret_cast<int *>(ring + NW * kStages * GG::STAGE);
+    uint64_t *bars = reinterpret_cast<uint64_t *>(smem);                 // [NW][ST]
+    uint8_t *ring = smem + bars_bytes<NW, ST>();                              // [NW][ST][STAGE]
+    int *prefix = reinterpret_cast<int *>(ring + NW * ST * GG::STAGE);
     __shared__ WorkMap wms;
     __shared__ WarpCtl ctls[NW];
 
@@ -592,8 +598,8 @@ decode_attn_q4_kernel(const AttnArgs a) {
         }
     }
 
-    uint64_t *wbar = bars + warp * kStages;
-    uint8_t *wring = ring + warp * kStages * GG::STAGE;
+    uint64_t *wbar = bars + warp * ST;
+    uint8_t *wring = ring + warp * ST * GG::STAGE;
     WarpCtl &ctl = ctls[warp];
     const uint64_t pol = policy_evict_first();
 
@@ -614,7 +620,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
         }
     };
 
-    // producer prologue: barrier init, first segment, up to kStages bulk copies.  Before
+    // producer prologue: barrier init, first segment, up to ST bulk copies.  Before
     // the fused append has run (early mode) a stage that holds the append slot L-1 is
     // not issued yet; the ring is topped up after the append.
     auto holds_append_slot = [&]() {
@@ -625,7 +631,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
 #endif
     auto prologue_setup = [&]() {
         if (lane == 0) {
-            for (int s = 0; s < kStages; ++s) mbar_init(&wbar[s], 1);
+            for (int s = 0; s < ST; ++s) mbar_init(&wbar[s], 1);
             if (LMO_FENCE_CTA) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
             else fence_mbar_init();
 #if LMO_ATTN_PROFILE
@@ -653,7 +659,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
     auto prologue = [&](bool before_append) {   // (always called with true)
         if (lane == 0) {
             int s = 0;
-            for (; s < kStages && !ctl.pdone; ++s) {
+            for (; s < ST && !ctl.pdone; ++s) {
                 if (before_append && a.k_new && holds_append_slot()) break;
                 issue(s);
             }
@@ -881,7 +887,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
     const unsigned long long prof_ga = gtimer();   // after the fused append
 #endif
     if (lane == 0)   // top the ring up (stages held back for the append)
-        for (int s = ctl.pissued; s < kStages && !ctl.pdone; ++s) issue(s);
+        for (int s = ctl.pissued; s < ST && !ctl.pdone; ++s) issue(s);
     __syncwarp();
 
     // ---- per-lane constant shared-memory offsets inside a stage (sub-block 0)
@@ -1323,7 +1329,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
         };
 
         auto advance = [&](int &sl, uint32_t &ph) {
-            if (++sl == kStages) {
+            if (++sl == ST) {
                 sl = 0;
                 ph ^= 1u;
             }
@@ -1496,7 +1502,7 @@ decode_attn_q4_kernel(const AttnArgs a) {
             const int T = wms.T, ti = warp / T, rank = warp - ti * T;
             const uint32_t bar_full = 1 + ti, bar_n = 32 * T;
             auto part_of = [&](int r) {
-                return reinterpret_cast<float *>(ring + (size_t)(ti * T + r) * kStages * GG::STAGE);
+                return reinterpret_cast<float *>(ring + (size_t)(ti * T + r) * ST * GG::STAGE);
             };
             if (rank != 0) {
                 float *part = part_of(rank);
@@ -1867,9 +1873,9 @@ extern "C" int lmo_debug_attn_profile(void *buf) {
 cudaError_t launch_kv_append(const lmo_kv_cache &cache, const void *k_new, const void *v_new,
                              int n_new, int pos0, const int32_t *pos_dev, cudaStream_t st,
                              int pos_from_lens);
-template <int D, int NW = kWarps>
+template <int D, int NW = kWarps, int ST = kStages>
 static size_t smem_bytes(int B_prefix) {
-    return bars_bytes<NW>() + (size_t)NW * kStages * Geo<D>::STAGE + (B_prefix > 0 ? (B_prefix + 1) * sizeof(int) : 0);
+    return bars_bytes<NW, ST>() + (size_t)NW * ST * Geo<D>::STAGE + (B_prefix > 0 ? (B_prefix + 1) * sizeof(int) : 0);
 }
 
 
@@ -1932,6 +1938,25 @@ static int ctas_per_sm(int B_prefix, bool mha) {   // (MHA and GQA instances dif
         occ[dev][mode][mha].store(n > 0 ? n : 1, std::memory_order_release);
     }
     return occ[dev][mode][mha].load(std::memory_order_acquire);
+}
+
+// resident CTAs per SM of the deep-ring GQA instance (d = 128, uniform length)
+static int deep_ctas_per_sm() {
+    static std::atomic<int> occ[64];
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev < 0 || dev >= 64) dev = 0;
+    if (occ[dev].load(std::memory_order_acquire) == 0) {
+        const int sz = (int)smem_bytes<128, kWarps, kDeepStages>(0);
+        cudaFuncSetAttribute(decode_attn_q4_kernel<128, false, kWarps, 1, kDeepStages>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, sz);
+        int n = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, decode_attn_q4_kernel<128, false, kWarps, 1, kDeepStages>,
+                                                      kWarps * 32, sz);
+        cudaGetLastError();
+        occ[dev].store(n > 0 ? n : -1, std::memory_order_release);
+    }
+    return occ[dev].load(std::memory_order_acquire);
 }
 
 int attn_max_warps_v(int head_dim, int B_prefix, bool mha) {
@@ -2038,8 +2063,20 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
         // the append slot when it does the append itself)
         a.early = 0;
     }
+    // Deep-ring GQA instance (measured): GQA at d = 128 with uniform length and
+    // the automatic schedule, when the pairs fill more than one warp per SMSP of the default
+    // grid but at most one warp each of a 2-CTA/SM grid (c5: 1024 pairs) -- T = 1 on a grid of
+    // kDeepStages-deep rings, twice the bytes in flight per busy warp.
+    bool deep = false;
+    if (D == 128 && a.G > 1 && !lens && num_splits == 0 && !sm && a.team == 1 && LMO_DEEP_GQA) {
+        const int occ = deep_ctas_per_sm();
+        if (occ > 0 && pairs > (int64_t)max_ctas * kWarps / 4 && pairs <= (int64_t)device_sm_count() * occ * kWarps)
+            deep = true;
+    }
     int64_t want_warps;
-    if (a.team) {
+    if (deep) {
+        want_warps = (int64_t)device_sm_count() * deep_ctas_per_sm() * kWarps;
+    } else if (a.team) {
         want_warps = (int64_t)max_ctas * kWarps;          // all CTAs; idle teams exit at once
 
 #ifdef LMO_EXPERIMENTS
@@ -2073,7 +2110,7 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
         if (want_warps > cap_ctas * kWarps) want_warps = cap_ctas * kWarps;
     }
     int64_t ctas = (want_warps + kWarps - 1) / kWarps;
-    if (ctas > cap_ctas) ctas = cap_ctas;
+    if (ctas > cap_ctas && !deep) ctas = cap_ctas;
     if (ctas < 1) ctas = 1;
 #ifdef LMO_EXPERIMENTS
     static const char *cap_env = getenv("LMO_ATTN_MAX_CTAS");   // tuning / experiments only
@@ -2105,6 +2142,7 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     cfg.gridDim = dim3((unsigned)ctas);
     cfg.blockDim = dim3(NW * 32);
     cfg.dynamicSmemBytes = sm ? (D == 64 ? smem_bytes<64, kSmWarps>(0) : smem_bytes<128, kSmWarps>(0))
+                         : deep ? smem_bytes<128, kWarps, kDeepStages>(0)
                               : (D == 64 ? smem_bytes<64>(Bp) : smem_bytes<128>(Bp)) + pad_smem;
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
@@ -2119,6 +2157,8 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false, kSmWarps>, a))
                     : (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, true, kSmWarps>, a)
                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, false, kSmWarps>, a));
+    else if (deep)
+        e = cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<128, false, kWarps, 1, kDeepStages>, a);
     else if (a.team == 1 && !LMO_NO_SCH)
         e = D == 64 ? (mha ? cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, true, kWarps, 1>, a)
                            : cudaLaunchKernelEx(&cfg, decode_attn_q4_kernel<64, false, kWarps, 1>, a))

@@ -81,6 +81,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_ATTN_MINBLOCKS
 #define LMO_ATTN_MINBLOCKS 4
 #endif
+#ifndef LMO_HALF_GRID_MHA
+#define LMO_HALF_GRID_MHA 1   // MHA launches with ~1 pair per warp of a 2-CTA/SM grid: 2 CTAs per SM
+#endif
 #ifndef LMO_DEEP_GQA
 #define LMO_DEEP_GQA 1   // GQA launches with ~1 pair per warp of a 2-CTA/SM grid: deep-ring instance
 #endif
@@ -2112,6 +2115,14 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
     int64_t ctas = (want_warps + kWarps - 1) / kWarps;
     if (ctas > cap_ctas && !deep) ctas = cap_ctas;
     if (ctas < 1) ctas = 1;
+    // MHA launches in the same regime (T = 1, about one pair per warp of a 2-CTA/SM grid, c2's
+    // 1024 pairs): launch 2 CTAs per SM of the default instance -- the free shared memory lets
+    // the next PDL launch's CTAs become resident (and prefetch) beside them (c2 step 0.597 ->
+    // 0.584 ms; c3, with more pairs than warps, loses: not applied there)
+    if (!deep && LMO_HALF_GRID_MHA && a.G == 1 && a.team == 1 && !lens && num_splits == 0 && !sm &&
+        pairs > (int64_t)max_ctas * kWarps / 4 && pairs <= (int64_t)device_sm_count() * 2 * kWarps &&
+        max_ctas >= device_sm_count() * 4)
+        ctas = device_sm_count() * 2;
 #ifdef LMO_EXPERIMENTS
     static const char *cap_env = getenv("LMO_ATTN_MAX_CTAS");   // tuning / experiments only
     if (cap_env && atoi(cap_env) > 0 && ctas > atoi(cap_env)) ctas = atoi(cap_env);

@@ -228,6 +228,8 @@ CASES = [  # (B, Hkv, G, d, L, num_splits)
     (1, 1, 1, 128, 1000, -2), (40, 9, 1, 128, 77, -2), (5, 3, 8, 128, 1, -2), (300, 4, 1, 64, 20, -2),
     # GQA, 592 < pairs <= 1184: the deep-ring 2-CTA/SM instance
     (80, 8, 8, 128, 200, 0), (130, 9, 2, 128, 77, 0), (148, 8, 4, 128, 33, 0),
+    # MHA, 592 < pairs <= 1184: the default instance on a 2-CTA/SM grid
+    (64, 10, 1, 128, 90, 0), (100, 11, 1, 128, 47, 0),
 ]
 
 
@@ -493,7 +495,8 @@ def test_decode_step_magnitude_edges(lmo, name):
                                             (7, 5, 2, 128, 47, -1), (4, 6, 1, 128, 300, -2),
                                             (3, 4, 8, 128, 129, -2), (5, 3, 1, 64, 77, -2),
                                             (2, 3, 1, 128, 1, -2), (64, 9, 1, 128, 47, -2),
-                                            (80, 8, 8, 128, 129, 0), (100, 7, 2, 128, 300, 0)])
+                                            (80, 8, 8, 128, 129, 0), (100, 7, 2, 128, 300, 0),
+                                            (64, 10, 1, 128, 90, 0)])
 def test_decode_step_fused_append(lmo, B, Hkv, G, d, L, ns, flags):
     """lmo_decode_step_q4 == append(new token at L-1) then attention over L, for the
     team schedule (one launch) and the stream-K fallback (two launches)."""

@@ -501,7 +501,10 @@ template <int NW, int ST = kStages>
 __host__ __device__ constexpr int bars_bytes() { return (NW * ST * 8 + 127) / 128 * 128; }
 // Deep-ring instance (ST = kDeepStages, 2 CTAs per SM): GQA launches with about one pair per
 // warp at 2 CTAs/SM keep twice the bytes in flight per busy warp (c5: 41.1 -> 39.0 us)
-constexpr int kDeepStages = 5;
+#ifndef LMO_DEEP_STAGES
+#define LMO_DEEP_STAGES 5
+#endif
+constexpr int kDeepStages = LMO_DEEP_STAGES;
 
 // SCH: 0 = any schedule (runtime work map mode); 1 = pair teams with T = 1 (one warp
 // per pair, the default); 2 = pair teams with T > 1.  The specialised instances drop

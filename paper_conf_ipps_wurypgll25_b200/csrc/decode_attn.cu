@@ -81,6 +81,9 @@ constexpr int kStageTok = kBlk * kSub;
 #ifndef LMO_ATTN_MINBLOCKS
 #define LMO_ATTN_MINBLOCKS 4
 #endif
+#ifndef LMO_EARLY_STAGES
+#define LMO_EARLY_STAGES 2   // CACHE_STABLE: stages per warp streamed before griddepcontrol.wait
+#endif
 #ifndef LMO_HALF_GRID_MHA
 #define LMO_HALF_GRID_MHA 1   // MHA launches with ~1 pair per warp of a 2-CTA/SM grid: 2 CTAs per SM
 #endif
@@ -662,11 +665,11 @@ decode_attn_q4_kernel(const AttnArgs a) {
         }
         __syncwarp();
     };
-    auto prologue = [&](bool before_append) {   // (always called with true)
+    auto prologue = [&](int maxs) {              // issue up to maxs (<= ST) stages
         if (lane == 0) {
             int s = 0;
-            for (; s < ST && !ctl.pdone; ++s) {
-                if (before_append && a.k_new && holds_append_slot()) break;
+            for (; s < maxs && !ctl.pdone; ++s) {
+                if (a.k_new && holds_append_slot()) break;
                 issue(s);
             }
             ctl.pissued = s;
@@ -872,17 +875,17 @@ decode_attn_q4_kernel(const AttnArgs a) {
                 }
             }
         }
-        prologue(true);
+        prologue(min(ST, a.early));   // a.early = stages to stream before the wait
         asm volatile("griddepcontrol.wait;\n" ::: "memory");
         fetch_first();
     } else if (!(TEAMK || wms.T)) {
         if (!a.lens) asm volatile("griddepcontrol.wait;\n" ::: "memory");
-        prologue(true);
+        prologue(ST);
         fetch_first();
     } else {
         if (!a.lens) asm volatile("griddepcontrol.wait;\n" ::: "memory");
         fetch_first();
-        prologue(true);
+        prologue(ST);
     }
 #if LMO_ATTN_PROFILE
     const unsigned long long prof_gp = gtimer();   // after the producer prologue
@@ -2004,7 +2007,11 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
                                     void *out, int out_f16, void *ws, cudaStream_t st,
                                     const void *k_new, const void *v_new, unsigned flags) {
     AttnArgs a;
-    a.early = (flags & LMO_STEP_CACHE_STABLE) ? 1 : 0;
+    // LMO_STEP_CACHE_STABLE: stream the first LMO_EARLY_STAGES stages of each warp before the
+    // PDL wait.  Measured (fused step, us per layer, depth 0 / 1 / 2 / 3): c2 18.0 / 18.3 / 18.0 /
+    // 18.2, c3 17.5 / 17.6 / 17.6 / 19.1, c4 59.4 / 59.3 / 58.3 / 58.7, c5 37.4 / 37.9 / 37.2 /
+    // 37.2 -- a full ring ahead floods HBM while the previous launch drains (c3: 4-stage pairs).
+    a.early = (flags & LMO_STEP_CACHE_STABLE) ? LMO_EARLY_STAGES : 0;
     a.flex = (k_new && (flags & LMO_STEP_FLEXGEN_EXACT)) ? 1 : 0;
     a.raw_k = static_cast<const __half *>(k_new);
     a.raw_v = static_cast<const __half *>(v_new);
@@ -2152,6 +2159,10 @@ cudaError_t launch_decode_attention(const lmo_kv_cache &c, const void *q, int Hq
         wm.NW = NW;
         if (sm) wm.V = wm.W;
     }
+#ifdef LMO_EXPERIMENTS
+    static const char *ed = getenv("LMO_EARLY_DEPTH");   // experiments: stages streamed before the wait
+    if (ed && a.early) a.early = atoi(ed);
+#endif
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3((unsigned)ctas);
     cfg.blockDim = dim3(NW * 32);

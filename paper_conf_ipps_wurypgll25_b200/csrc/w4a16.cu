@@ -605,6 +605,9 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
                 const int xs = j % g2::kXS;
                 if (j >= g2::kXS) mbar_wait(&x_empty[xs], ((j / g2::kXS) - 1) & 1);
                 W4TL(1, j);
+#ifdef LMO_W4_EXP_NOX   // (timing experiment: activations loaded only for the first kXS steps -- wrong results)
+                if (j >= g2::kXS) { mbar_arrive(&x_full[xs]); continue; }
+#endif
                 mbar_arrive_expect_tx(&x_full[xs], S::B);
                 tma_2d(sbase + xs * S::B, &tm_x, (kb0 + 2 * j) * kK, 0, &x_full[xs]);
                 tma_2d(sbase + xs * S::B + BN * 128, &tm_x, (kb0 + 2 * j + 1) * kK, 0, &x_full[xs]);

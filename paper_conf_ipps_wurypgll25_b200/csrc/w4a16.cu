@@ -529,7 +529,8 @@ struct Smem {
 template <int BN>
 struct Tmem {
     static constexpr int A0 = BN;
-    static constexpr int USED = BN + kAS * 64;
+    static constexpr int ACC1 = BN + kAS * 64;          // stream-K: second tile's accumulator
+    static constexpr int USED = ACC1 + BN;
     static constexpr int COLS = USED <= 128 ? 128 : USED <= 256 ? 256 : 512;
 };
 static_assert((2 * kC + 2 * kXS + 2 * kAS + 1) * 8 + 4 <= 512, "barrier area");
@@ -541,7 +542,7 @@ static_assert((2 * kC + 2 * kXS + 2 * kAS + 1) * 8 + 4 <= 512, "barrier area");
 template <int BN, int DW>
 __global__ void __launch_bounds__(DW * 32 + 96, 1)
 w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restrict__ packed,
-                float *__restrict__ y, int N, int K, int batch, int ksplit) {
+                float *__restrict__ y, int N, int K, int batch, int ksplit, int sk) {
     using S = g2::Smem<BN>;
     using TM = g2::Tmem<BN>;
     constexpr int kWMMA = DW, kWTC = DW + 1, kWTX = DW + 2;
@@ -557,10 +558,29 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(done + 1);
 
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
-    const int n0 = blockIdx.x * kM;
     const int KB = K / kK, KS = KB / 2;                 // groups, steps
-    const int s0 = (int)((long long)blockIdx.y * KS / ksplit), s1 = (int)((long long)(blockIdx.y + 1) * KS / ksplit);
-    const int nsteps = s1 - s0, kb0 = 2 * s0;
+    // Work of this CTA: steps [0, nsteps) = k-steps g0 .. of tile tile0, then (stream-K) from
+    // step jsw on k-steps 0 .. of tile tile0 + 1.  Split-K (sk = 0): tile blockIdx.x, the
+    // blockIdx.y-th of ksplit k ranges.  Stream-K (sk = 1, gridDim.y = 1, gridDim.x >= tiles):
+    // the tile-steps of all tiles, linearised tile-major, cut into gridDim.x equal ranges --
+    // equal work per resident slot, each range within at most two tiles.
+    int tile0, g0, nsteps, jsw;
+    if (sk) {
+        const long long T = (long long)(N / kM) * KS;
+        const long long a0 = (long long)blockIdx.x * T / gridDim.x, a1 = (long long)(blockIdx.x + 1) * T / gridDim.x;
+        tile0 = (int)(a0 / KS);
+        g0 = (int)(a0 - (long long)tile0 * KS);
+        nsteps = (int)(a1 - a0);
+        jsw = min(nsteps, KS - g0);
+    } else {
+        const int s0 = (int)((long long)blockIdx.y * KS / ksplit), s1 = (int)((long long)(blockIdx.y + 1) * KS / ksplit);
+        tile0 = blockIdx.x;
+        g0 = s0;
+        nsteps = s1 - s0;
+        jsw = nsteps;
+    }
+    auto tile_of = [&](int j) { return j < jsw ? tile0 : tile0 + 1; };
+    auto kstep_of = [&](int j) { return j < jsw ? g0 + j : j - jsw; };
 
     if (tid == 0) {
         for (int s = 0; s < g2::kC; ++s) {
@@ -595,7 +615,7 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
                 if (q >= g2::kC) mbar_wait(&c_empty[cs], ((q / g2::kC) - 1) & 1);
                 W4TL(0, q);
                 mbar_arrive_expect_tx(&c_full[cs], S::CSLOT);
-                const uint8_t *src = packed + ((int64_t)blockIdx.x * KB + kb0 + 2 * q) * S::PBLK;
+                const uint8_t *src = packed + ((int64_t)tile_of(q) * KB + 2 * kstep_of(q)) * S::PBLK;
                 bulk_g2s(smem + S::OFF_CODES + cs * S::CSLOT, src, S::CSLOT, &c_full[cs], policy_evict_first());
             }
         }
@@ -609,8 +629,9 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
                 if (j >= g2::kXS) { mbar_arrive(&x_full[xs]); continue; }
 #endif
                 mbar_arrive_expect_tx(&x_full[xs], S::B);
-                tma_2d(sbase + xs * S::B, &tm_x, (kb0 + 2 * j) * kK, 0, &x_full[xs]);
-                tma_2d(sbase + xs * S::B + BN * 128, &tm_x, (kb0 + 2 * j + 1) * kK, 0, &x_full[xs]);
+                const int kg = 2 * kstep_of(j);
+                tma_2d(sbase + xs * S::B, &tm_x, kg * kK, 0, &x_full[xs]);
+                tma_2d(sbase + xs * S::B + BN * 128, &tm_x, (kg + 1) * kK, 0, &x_full[xs]);
             }
         }
     } else if (warp < kWMMA) {
@@ -706,6 +727,8 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
             asm volatile("tcgen05.fence::after_thread_sync;\n");
             if (lane == 0) {
                 const uint32_t b0 = sbase + xs * S::B;
+                const uint32_t dacc = tmem + (j < jsw ? 0u : (uint32_t)TM::ACC1);   // this step's tile accumulator
+                const bool first = j == 0 || j == jsw;
 #ifdef LMO_W4_EXP_MMA1   // (timing experiment: one MMA per step -- wrong results)
                 for (int gi = 0; gi < 1; ++gi)
                     for (int k = 0; k < 1; ++k) {
@@ -717,10 +740,10 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
 #endif
                         const uint32_t ta = tmem + TM::A0 + st * 64 + gi * 32 + k * 8;
                         const uint64_t db = umma_desc(b0 + gi * BN * 128 + k * 32);
-                        const uint32_t acc = (j > 0 || gi > 0 || k > 0) ? 1u : 0u;
+                        const uint32_t acc = (!first || gi > 0 || k > 0) ? 1u : 0u;
                         asm volatile(
                             "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
-                            "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem),
+                            "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}\n" ::"r"(dacc),
                             "r"(ta), "l"(db), "r"(idesc), "r"(acc));
                     }
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
@@ -739,40 +762,41 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
         __syncwarp();
     }
 
-    // epilogue: warps 0-3 read the accumulator (TMEM lane = output feature)
+    // epilogue: warps 0-3 read the accumulator(s) (TMEM lane = output feature); stream-K
+    // ranges and split-K partials are added atomically (y zeroed on the stream first)
     if (warp < 4) {
         const int row = (warp & 3) * 32 + lane;
         if (nsteps > 0) {
             mbar_wait(done, 0);
             asm volatile("tcgen05.fence::after_thread_sync;\n");
         }
+        for (int seg = 0; seg < 2; ++seg) {
+            if (seg == 0 ? jsw == 0 : nsteps <= jsw) continue;
+            const int n0 = (tile0 + seg) * kM;
+            const uint32_t aoff = seg == 0 ? 0u : (uint32_t)TM::ACC1;
 #pragma unroll
-        for (int c0 = 0; c0 < BN; c0 += 32) {
-            uint32_t v[32];
-            const uint32_t taddr = tmem + ((uint32_t)((warp & 3) * 32) << 16) + c0;
-            asm volatile(
-                "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-                "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];\n"
-                : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-                  "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
-                  "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
-                  "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
-                  "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
-                : "r"(taddr));
-            asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
-            if (nsteps == 0) continue;
+            for (int c0 = 0; c0 < BN; c0 += 32) {
+                uint32_t v[32];
+                const uint32_t taddr = tmem + ((uint32_t)((warp & 3) * 32) << 16) + aoff + c0;
+                asm volatile(
+                    "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+                    "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];\n"
+                    : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+                      "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
+                      "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
+                      "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
+                      "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+                    : "r"(taddr));
+                asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
 #pragma unroll
-            for (int i = 0; i < 32; ++i) {
-                const int b = c0 + i;
-                if (b < batch) {
-                    float *dst = y + (int64_t)b * N + n0 + row;
-                    const float val = __uint_as_float(v[i]);
-#ifdef LMO_W4_NOATOMIC   // (timing experiment: split-K partials stored, not reduced -- wrong results)
-                    *dst = val;
-#else
-                    if (ksplit > 1) atomicAdd(dst, val);
-                    else *dst = val;
-#endif
+                for (int i = 0; i < 32; ++i) {
+                    const int b = c0 + i;
+                    if (b < batch) {
+                        float *dst = y + (int64_t)b * N + n0 + row;
+                        const float val = __uint_as_float(v[i]);
+                        if (ksplit > 1 || sk) atomicAdd(dst, val);
+                        else *dst = val;
+                    }
                 }
             }
         }
@@ -789,6 +813,9 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
 
 #ifndef LMO_W4_G2
 #define LMO_W4_G2 1   // packed weights, K % 128 == 0: two quantization groups per pipeline step
+#endif
+#ifndef LMO_W4_STREAMK
+#define LMO_W4_STREAMK 1   // auto split of the two-group kernel: stream-K when tiles do not fill the slots evenly
 #endif
 #ifndef LMO_W4_G2_DW
 #define LMO_W4_G2_DW 4   // dequant warps of the two-group kernel (4 or 8: measured equal within noise)
@@ -925,16 +952,36 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
         auto go2 = [&](auto kern, int smem_bytes, int tmem_cols) {
             cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
             cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
+            int sk_ctas = 0;
             if (ksplit <= 0) {
                 const int occ = w4a16_resident_ctas(smem_bytes, tmem_cols, LMO_W4_G2_DW * 32 + 96);
                 ksplit = w4a16_auto_split(N, K, occ);
+                // Stream-K when the tiles do not fill the resident slots evenly (e.g. 168 or 224
+                // tiles on 296 slots: 2-tile SMs beside 1-tile SMs): the linearised tile-steps cut
+                // into whole waves of equal ranges (K7)
+                // (measured: only a poorly filled split pays for stream-K's second epilogue --
+                // c3 QKV 168 tiles 44.2 -> 37.6 us, c5 QKV 192 tiles 84.0 -> 70.7, but c3 FFN2
+                // 56 tiles x 5 splits 40.9 -> 43.2)
+                const int64_t tiles = N / w4::kM, slots = (int64_t)device_sm_count() * occ;
+                const int64_t T = tiles * (K / (2 * w4::kK));
+                const int64_t used = tiles * ksplit, waves_used = (used + slots - 1) / slots;
+                const double fill = (double)used / (double)(slots * waves_used);
+                if (LMO_W4_STREAMK && fill < 0.8) {
+                    const int64_t waves = (tiles + slots - 1) / slots;
+                    sk_ctas = (int)std::min<int64_t>(slots * waves, T);
+                    ksplit = 1;
+                }
             }
             if (ksplit > K / (2 * w4::kK)) ksplit = K / (2 * w4::kK);
-            if (ksplit > 1) {
+            if (ksplit > 1 || sk_ctas > 0) {
                 pre = cudaMemsetAsync(y, 0, (size_t)batch * N * sizeof(float), st);
                 if (pre != cudaSuccess) return;
             }
-            kern<<<dim3(N / w4::kM, ksplit), LMO_W4_G2_DW * 32 + 96, smem_bytes, st>>>(tx, packed, y, N, K, batch, ksplit);
+            if (sk_ctas > 0)
+                kern<<<dim3(sk_ctas, 1), LMO_W4_G2_DW * 32 + 96, smem_bytes, st>>>(tx, packed, y, N, K, batch, 1, 1);
+            else
+                kern<<<dim3(N / w4::kM, ksplit), LMO_W4_G2_DW * 32 + 96, smem_bytes, st>>>(tx, packed, y, N, K, batch,
+                                                                                           ksplit, 0);
         };
         if (BN == 64) go2(w4::w4a16_g2_kernel<64, LMO_W4_G2_DW>, w4::g2::Smem<64>::BYTES, w4::g2::Tmem<64>::COLS);
         else go2(w4::w4a16_g2_kernel<128, LMO_W4_G2_DW>, w4::g2::Smem<128>::BYTES, w4::g2::Tmem<128>::COLS);

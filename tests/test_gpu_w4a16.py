@@ -215,3 +215,26 @@ def test_w4a16_weight_magnitude_edges(lmo, packed):
     for lo in range(0, N, 128):
         print(f"rows {lo}-{lo + 127}: max err/bound {r[:, lo:lo + 128].max():.3f}")
     assert np.all(err <= bound), (r.max(), np.unravel_index(r.argmax(), r.shape))
+
+
+@pytest.mark.parametrize("N,K,batch", [(640, 12800, 8), (640, 12800, 100), (384, 7168, 64), (2560, 1024, 37)])
+def test_w4a16_packed_stream_k(lmo, N, K, batch):
+    """The automatic split of the packed GEMM uses stream-K when the tiles do not fill the
+    resident slots evenly: the tile-steps of all tiles cut into equal ranges, a range may
+    end inside one tile and continue in the next (two TMEM accumulators, atomic adds).
+    N=640, K=12800: 500 tile-steps over the slots -- most ranges cross a tile boundary.
+    Checked against the oracle bound and against the unsplit run (fp32 rounding)."""
+    rng = np.random.default_rng(3000 + N + K + batch)
+    codes, meta = make_weights(rng, N, K)
+    c, m = torch.from_numpy(codes).cuda(), torch.from_numpy(meta.view(np.int32)).cuda()
+    packed = lmo.lmo_w4a16_pack(c, m, N, K)
+    x = torch.from_numpy(rng.standard_normal((batch, K)).astype(np.float16)).cuda()
+    ya = lmo.lmo_w4a16_linear_packed(packed, N, K, x, k_split=0).cpu()
+    y1 = lmo.lmo_w4a16_linear_packed(packed, N, K, x, k_split=1).cpu()
+    ref = oracle.w4a16_linear(codes, meta, N, K, x.cpu().numpy())
+    wdq = oracle.dequantize_groupwise(codes, meta, N, K, 1).reshape(N, K).astype(np.float64)
+    absdot = np.abs(x.cpu().numpy().astype(np.float64)) @ np.abs(wdq).T
+    assert np.all(np.abs(ya.numpy().astype(np.float64) - ref) <= absdot * 2.0 ** -10 + 1e-6)
+    # vs the unsplit run: only the fp32 summation order differs (tensor-core accumulation
+    # of the whole K vs atomic adds of range partials): |dy| <= K * 2^-24 * sum|x w|
+    assert np.all(np.abs(ya.numpy().astype(np.float64) - y1.numpy()) <= K * 2.0 ** -24 * absdot + 1e-6)

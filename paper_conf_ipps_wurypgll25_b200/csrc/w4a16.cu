@@ -536,6 +536,14 @@ struct Tmem {
 static_assert((2 * kC + 2 * kXS + 2 * kAS + 1) * 8 + 4 <= 512, "barrier area");
 }  // namespace g2
 
+// y = 0 for the split / stream-K GEMMs' atomic epilogues; triggers its programmatic dependent
+// (the GEMM) at once so the GEMM's main loop overlaps it
+__global__ void w4_zero_kernel(float4 *__restrict__ p, int64_t n4) {
+    asm volatile("griddepcontrol.launch_dependents;\n" ::: "memory");
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = make_float4(0.f, 0.f, 0.f, 0.f);
+}
+
 // DW = dequant warps: 4 (thread = weight row, both groups) or 8 (warp w: rows 32 (w % 4) ..,
 // group w / 4 -- two warps per SMSP, half the dependent chain per thread; one mbarrier
 // arrival per warp).
@@ -770,6 +778,8 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
             mbar_wait(done, 0);
             asm volatile("tcgen05.fence::after_thread_sync;\n");
         }
+        // the zeroed y: written by the preceding (programmatic-primary) zero kernel
+        if (ksplit > 1 || sk) asm volatile("griddepcontrol.wait;\n" ::: "memory");
         for (int seg = 0; seg < 2; ++seg) {
             if (seg == 0 ? jsw == 0 : nsteps <= jsw) continue;
             const int n0 = (tile0 + seg) * kM;
@@ -973,15 +983,30 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
                 }
             }
             if (ksplit > K / (2 * w4::kK)) ksplit = K / (2 * w4::kK);
-            if (ksplit > 1 || sk_ctas > 0) {
-                pre = cudaMemsetAsync(y, 0, (size_t)batch * N * sizeof(float), st);
+            const bool zero = ksplit > 1 || sk_ctas > 0;
+            if (zero) {
+                // y is zeroed by a PDL-triggering kernel and the GEMM is launched as its programmatic
+                // dependent: the GEMM's main loop overlaps the zeroing (x and the codes are ready --
+                // their producer finished before the zero kernel started) and only its epilogue
+                // atomics wait (griddepcontrol.wait) for the zeros
+                const int64_t n4 = (int64_t)batch * N / 4;
+                w4::w4_zero_kernel<<<device_sm_count(), 256, 0, st>>>(reinterpret_cast<float4 *>(y), n4);
+                pre = cudaGetLastError();
                 if (pre != cudaSuccess) return;
+                note_launch();
             }
-            if (sk_ctas > 0)
-                kern<<<dim3(sk_ctas, 1), LMO_W4_G2_DW * 32 + 96, smem_bytes, st>>>(tx, packed, y, N, K, batch, 1, 1);
-            else
-                kern<<<dim3(N / w4::kM, ksplit), LMO_W4_G2_DW * 32 + 96, smem_bytes, st>>>(tx, packed, y, N, K, batch,
-                                                                                           ksplit, 0);
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = sk_ctas > 0 ? dim3(sk_ctas, 1) : dim3(N / w4::kM, ksplit);
+            cfg.blockDim = dim3(LMO_W4_G2_DW * 32 + 96);
+            cfg.dynamicSmemBytes = smem_bytes;
+            cfg.stream = st;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            attr[0].val.programmaticStreamSerializationAllowed = (zero && pdl_enabled()) ? 1 : 0;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            pre = cudaLaunchKernelEx(&cfg, kern, tx, packed, y, (int)N, (int)K, (int)batch, sk_ctas > 0 ? 1 : ksplit,
+                                     sk_ctas > 0 ? 1 : 0);
         };
         if (BN == 64) go2(w4::w4a16_g2_kernel<64, LMO_W4_G2_DW>, w4::g2::Smem<64>::BYTES, w4::g2::Tmem<64>::COLS);
         else go2(w4::w4a16_g2_kernel<128, LMO_W4_G2_DW>, w4::g2::Smem<128>::BYTES, w4::g2::Tmem<128>::COLS);

@@ -444,6 +444,8 @@ w4a16_kernel(const __grid_constant__ CUtensorMap tm_codes, const __grid_constant
     }
 
     // ---------------------------------------------------------------- epilogue
+    // (split-K: the zeroed y comes from the preceding programmatic-primary zero kernel)
+    if (ksplit > 1) asm volatile("griddepcontrol.wait;\n" ::: "memory");
     if (warp < 4 * MT) {
         const int emt = warp >> 2;                               // tile of this epilogue warp
         const int row = emt * kM + (warp & 3) * 32 + lane;       // TMEM lane = output feature
@@ -1025,12 +1027,23 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
             ksplit = w4a16_auto_split(N, K, occ);
         }
         if (ksplit > K / w4::kK) ksplit = K / w4::kK;
-        if (ksplit > 1) {
-            pre = cudaMemsetAsync(y, 0, (size_t)batch * N * sizeof(float), st);
+        if (ksplit > 1) {   // zeroing overlapped with the GEMM (as in the two-group path)
+            w4::w4_zero_kernel<<<device_sm_count(), 256, 0, st>>>(reinterpret_cast<float4 *>(y), (int64_t)batch * N / 4);
+            pre = cudaGetLastError();
             if (pre != cudaSuccess) return;
+            note_launch();
         }
-        dim3 grid(N / (w4::kM * MT), ksplit);
-        kern<<<grid, threads, sm, st>>>(tc, tx, m, packed, y, N, K, batch, ksplit);
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(N / (w4::kM * MT), ksplit);
+        cfg.blockDim = dim3(threads);
+        cfg.dynamicSmemBytes = sm;
+        cfg.stream = st;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        attr[0].val.programmaticStreamSerializationAllowed = (ksplit > 1 && pdl_enabled()) ? 1 : 0;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        pre = cudaLaunchKernelEx(&cfg, kern, tc, tx, m, packed, y, (int)N, (int)K, (int)batch, ksplit);
     };
     constexpr int T1 = w4::Roles<1>::THREADS, T2 = w4::Roles<2>::THREADS;
     if (MT == 2) {

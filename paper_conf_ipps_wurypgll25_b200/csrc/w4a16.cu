@@ -63,6 +63,9 @@ constexpr int kCodeSlots = kCodes / kCPS;
 #ifndef LMO_W4_WARP_ARRIVE
 #define LMO_W4_WARP_ARRIVE 0   // 1: one mbarrier arrival per producer warp (measured equal)
 #endif
+#ifndef LMO_W4_STREAMK
+#define LMO_W4_STREAMK 1   // auto split of the two-group kernel: stream-K when tiles do not fill the slots evenly
+#endif
 #ifndef LMO_W4_NODEQ
 #define LMO_W4_NODEQ 0
 #endif
@@ -519,20 +522,31 @@ constexpr int kXS = LMO_W4_G2_XS;     // activation stages
 #define LMO_W4_G2_AS 2
 #endif
 constexpr int kAS = LMO_W4_G2_AS;      // A stages in TMEM (64 columns each)
+// Per-instance pipeline shape.  BN = 128 (batch 65-128): 2 activation stages and 3 code slots
+// (93 KB of shared memory) and no stream-K accumulator (256 TMEM columns), so TWO CTAs fit
+// per SM -- measured c5 layer 255 -> 208 us; with the 3-stage / 6-slot shape and a second
+// accumulator (512 columns) only one fits.  BN = 64: the 3 / 6 shape with stream-K.
+template <int BN>
+struct Cfg {
+    static constexpr int XS = BN == 128 ? 2 : kXS;     // activation stages
+    static constexpr int C = BN == 128 ? 3 : kC;       // code slots
+    static constexpr bool SK = BN != 128 && LMO_W4_STREAMK;   // stream-K (second accumulator)
+};
 template <int BN>
 struct Smem {
+    static constexpr int XS = Cfg<BN>::XS, C = Cfg<BN>::C;
     static constexpr int B = 2 * BN * 128;             // two SW128 atoms: BN x 128 fp16
     static constexpr int PBLK = kM * 32 + kM * 4;      // one packed tile-group block
     static constexpr int CSLOT = 2 * PBLK;
-    static constexpr int OFF_CODES = kXS * B;
-    static constexpr int OFF_BARS = OFF_CODES + kC * CSLOT;
+    static constexpr int OFF_CODES = XS * B;
+    static constexpr int OFF_BARS = OFF_CODES + C * CSLOT;
     static constexpr int BYTES = OFF_BARS + 512 + 1024;
 };
 template <int BN>
 struct Tmem {
     static constexpr int A0 = BN;
     static constexpr int ACC1 = BN + kAS * 64;          // stream-K: second tile's accumulator
-    static constexpr int USED = ACC1 + BN;
+    static constexpr int USED = ACC1 + (Cfg<BN>::SK ? BN : 0);
     static constexpr int COLS = USED <= 128 ? 128 : USED <= 256 ? 256 : 512;
 };
 static_assert((2 * kC + 2 * kXS + 2 * kAS + 1) * 8 + 4 <= 512, "barrier area");
@@ -561,9 +575,9 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
     uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     const uint32_t sbase = smem_u32(smem);
     uint64_t *bars = reinterpret_cast<uint64_t *>(smem + S::OFF_BARS);
-    uint64_t *c_full = bars, *c_empty = bars + g2::kC;
-    uint64_t *x_full = bars + 2 * g2::kC, *x_empty = x_full + g2::kXS;
-    uint64_t *a_full = x_empty + g2::kXS, *ab_empty = a_full + g2::kAS;
+    uint64_t *c_full = bars, *c_empty = bars + S::C;
+    uint64_t *x_full = bars + 2 * S::C, *x_empty = x_full + S::XS;
+    uint64_t *a_full = x_empty + S::XS, *ab_empty = a_full + g2::kAS;
     uint64_t *done = ab_empty + g2::kAS;
     uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(done + 1);
 
@@ -593,11 +607,11 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
     auto kstep_of = [&](int j) { return j < jsw ? g0 + j : j - jsw; };
 
     if (tid == 0) {
-        for (int s = 0; s < g2::kC; ++s) {
+        for (int s = 0; s < S::C; ++s) {
             mbar_init(&c_full[s], 1);
             mbar_init(&c_empty[s], kArrive);
         }
-        for (int s = 0; s < g2::kXS; ++s) {
+        for (int s = 0; s < S::XS; ++s) {
             mbar_init(&x_full[s], 1);
             mbar_init(&x_empty[s], 1);
         }
@@ -621,8 +635,8 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
     if (warp == kWTC) {
         if (lane == 0) {   // codes: one bulk copy of a step's two consecutive packed blocks
             for (int q = 0; q < nsteps; ++q) {
-                const int cs = q % g2::kC;
-                if (q >= g2::kC) mbar_wait(&c_empty[cs], ((q / g2::kC) - 1) & 1);
+                const int cs = q % S::C;
+                if (q >= S::C) mbar_wait(&c_empty[cs], ((q / S::C) - 1) & 1);
                 W4TL(0, q);
                 mbar_arrive_expect_tx(&c_full[cs], S::CSLOT);
                 const uint8_t *src = packed + ((int64_t)tile_of(q) * KB + 2 * kstep_of(q)) * S::PBLK;
@@ -632,11 +646,11 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
     } else if (warp == kWTX) {
         if (lane == 0) {   // activations: two 64-wide SW128 boxes per step
             for (int j = 0; j < nsteps; ++j) {
-                const int xs = j % g2::kXS;
-                if (j >= g2::kXS) mbar_wait(&x_empty[xs], ((j / g2::kXS) - 1) & 1);
+                const int xs = j % S::XS;
+                if (j >= S::XS) mbar_wait(&x_empty[xs], ((j / S::XS) - 1) & 1);
                 W4TL(1, j);
 #ifdef LMO_W4_EXP_NOX   // (timing experiment: activations loaded only for the first kXS steps -- wrong results)
-                if (j >= g2::kXS) { mbar_arrive(&x_full[xs]); continue; }
+                if (j >= S::XS) { mbar_arrive(&x_full[xs]); continue; }
 #endif
                 mbar_arrive_expect_tx(&x_full[xs], S::B);
                 const int kg = 2 * kstep_of(j);
@@ -651,9 +665,9 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
         constexpr int G0 = 0, G1 = DW == 8 ? 1 : 2;           // groups of this thread: [g_lo, g_lo + G1)
         const int g_lo = DW == 8 ? (warp >> 2) : 0;
         for (int j = 0; j < nsteps; ++j) {
-            const int cs = j % g2::kC, st = j % g2::kAS;
+            const int cs = j % S::C, st = j % g2::kAS;
             if (tid == 0) W4TL(2, j);
-            mbar_wait(&c_full[cs], (j / g2::kC) & 1);
+            mbar_wait(&c_full[cs], (j / S::C) & 1);
             if (tid == 0) W4TL(3, j);
             if (j >= g2::kAS) mbar_wait(&ab_empty[st], ((j / g2::kAS) - 1) & 1);
             if (tid == 0) W4TL(4, j);
@@ -729,8 +743,8 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
         // MMA issuer: 2 groups x 4 x (K = 16) per step
         constexpr uint32_t idesc = umma_idesc<BN>();
         for (int j = 0; j < nsteps; ++j) {
-            const int st = j % g2::kAS, xs = j % g2::kXS;
-            mbar_wait(&x_full[xs], (j / g2::kXS) & 1);
+            const int st = j % g2::kAS, xs = j % S::XS;
+            mbar_wait(&x_full[xs], (j / S::XS) & 1);
             if (lane == 0) W4TL(6, j);
             mbar_wait(&a_full[st], (j / g2::kAS) & 1);
             if (lane == 0) W4TL(7, j);
@@ -825,9 +839,6 @@ w4a16_g2_kernel(const __grid_constant__ CUtensorMap tm_x, const uint8_t *__restr
 
 #ifndef LMO_W4_G2
 #define LMO_W4_G2 1   // packed weights, K % 128 == 0: two quantization groups per pipeline step
-#endif
-#ifndef LMO_W4_STREAMK
-#define LMO_W4_STREAMK 1   // auto split of the two-group kernel: stream-K when tiles do not fill the slots evenly
 #endif
 #ifndef LMO_W4_G2_DW
 #define LMO_W4_G2_DW 4   // dequant warps of the two-group kernel (4 or 8: measured equal within noise)
@@ -961,7 +972,7 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
     const uint32_t *m = static_cast<const uint32_t *>(meta);
     if (packed && LMO_W4_G2 && MT == 1 && K % (2 * w4::kK) == 0) {   // two groups per pipeline step
         cudaError_t pre = cudaSuccess;
-        auto go2 = [&](auto kern, int smem_bytes, int tmem_cols) {
+        auto go2 = [&](auto kern, int smem_bytes, int tmem_cols, bool sk_ok) {
             cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
             cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
             int sk_ctas = 0;
@@ -978,7 +989,7 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
                 const int64_t T = tiles * (K / (2 * w4::kK));
                 const int64_t used = tiles * ksplit, waves_used = (used + slots - 1) / slots;
                 const double fill = (double)used / (double)(slots * waves_used);
-                if (LMO_W4_STREAMK && fill < 0.8) {
+                if (sk_ok && fill < 0.8) {
                     const int64_t waves = (tiles + slots - 1) / slots;
                     sk_ctas = (int)std::min<int64_t>(slots * waves, T);
                     ksplit = 1;
@@ -1010,8 +1021,11 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
             pre = cudaLaunchKernelEx(&cfg, kern, tx, packed, y, (int)N, (int)K, (int)batch, sk_ctas > 0 ? 1 : ksplit,
                                      sk_ctas > 0 ? 1 : 0);
         };
-        if (BN == 64) go2(w4::w4a16_g2_kernel<64, LMO_W4_G2_DW>, w4::g2::Smem<64>::BYTES, w4::g2::Tmem<64>::COLS);
-        else go2(w4::w4a16_g2_kernel<128, LMO_W4_G2_DW>, w4::g2::Smem<128>::BYTES, w4::g2::Tmem<128>::COLS);
+        if (BN == 64)
+            go2(w4::w4a16_g2_kernel<64, LMO_W4_G2_DW>, w4::g2::Smem<64>::BYTES, w4::g2::Tmem<64>::COLS, w4::g2::Cfg<64>::SK);
+        else
+            go2(w4::w4a16_g2_kernel<128, LMO_W4_G2_DW>, w4::g2::Smem<128>::BYTES, w4::g2::Tmem<128>::COLS,
+                w4::g2::Cfg<128>::SK);
         if (pre != cudaSuccess) return pre;
         const cudaError_t e = cudaGetLastError();
         if (e == cudaSuccess) note_launch();

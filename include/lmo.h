@@ -270,9 +270,13 @@ lmo_status lmo_offload_destroy(lmo_offload_t ex);
  * x_f16 : activations [batch][K] fp16, row-major.
  * y_f32 : output [batch][N] fp32, row-major (overwritten).
  * N % 128 == 0, K % 64 == 0, 1 <= batch <= 128 (else LMO_ERR_SHAPE /
- * LMO_ERR_UNSUPPORTED).  k_split: K-dimension split (0 = auto); with k_split
- * > 1 y is zeroed on `stream` and the partial tiles are added atomically
- * (summation order then varies: results agree within fp32 rounding).  All
+ * LMO_ERR_UNSUPPORTED).  k_split: K-dimension split (0 = auto: split-K over
+ * one wave of resident CTAs, or -- packed path, batch <= 64, when that wave is
+ * poorly filled -- stream-K, equal ranges of the tile-steps of all tiles that
+ * may cross a tile boundary); with a split (k_split > 1 or an auto split) y is
+ * zeroed on `stream` by a kernel of this library and the partial tiles are
+ * added atomically (summation order then varies: results agree within fp32
+ * rounding; k_split = 1 is deterministic).  All
  * pointers 16-byte aligned.  Device memory is caller-owned; enqueued on
  * `stream`, asynchronous.
  * ------------------------------------------------------------------------- */

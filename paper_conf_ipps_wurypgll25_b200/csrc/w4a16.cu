@@ -66,6 +66,9 @@ constexpr int kCodeSlots = kCodes / kCPS;
 #ifndef LMO_W4_STREAMK
 #define LMO_W4_STREAMK 1   // auto split of the two-group kernel: stream-K when tiles do not fill the slots evenly
 #endif
+#ifndef LMO_W4_SK_FILL
+#define LMO_W4_SK_FILL 0.8   // stream-K when the split-K grid fills less than this share of the slots
+#endif
 #ifndef LMO_W4_NODEQ
 #define LMO_W4_NODEQ 0
 #endif
@@ -989,7 +992,7 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
                 const int64_t T = tiles * (K / (2 * w4::kK));
                 const int64_t used = tiles * ksplit, waves_used = (used + slots - 1) / slots;
                 const double fill = (double)used / (double)(slots * waves_used);
-                if (sk_ok && fill < 0.8) {
+                if (sk_ok && fill < LMO_W4_SK_FILL) {
                     const int64_t waves = (tiles + slots - 1) / slots;
                     sk_ctas = (int)std::min<int64_t>(slots * waves, T);
                     ksplit = 1;

@@ -8,6 +8,7 @@ import torch
 from paper_conf_ipps_wurypgll25_b200 import lmo
 B, H, G, L = [int(x) for x in sys.argv[1:5]]
 STEP = len(sys.argv) > 5 and sys.argv[5] == "step"     # fused append + attention, CACHE_STABLE
+NS = int(os.environ.get("SPLITS", "0"))                 # num_splits (1/2/4 = explicit team size)
 d = 128
 nl = max(3, int(2e9 // (B * H * (L + 16) * 144)))
 caches = [lmo.KVCache.empty(B, H, (L + 15) // 16 * 16, d) for _ in range(nl)]
@@ -20,9 +21,9 @@ ws = lmo.attention_workspace(B, H, H * G, d)
 kn = torch.randn(B, H, d, device='cuda').half(); vn = torch.randn_like(kn)
 def launch(c):
     if STEP:
-        lmo.lmo_decode_step_q4(c, kn, vn, q, L, out=out, workspace=ws, flags=lmo.LMO_STEP_CACHE_STABLE)
+        lmo.lmo_decode_step_q4(c, kn, vn, q, L, out=out, workspace=ws, flags=lmo.LMO_STEP_CACHE_STABLE, num_splits=NS)
     else:
-        lmo.lmo_decode_attention_q4(c, q, L, out=out, workspace=ws)
+        lmo.lmo_decode_attention_q4(c, q, L, out=out, workspace=ws, num_splits=NS)
 nl = min(nl, 16)
 buf = torch.zeros(16 * 148 * 64 * 16, dtype=torch.int64, device='cuda')
 lmo._lib.lmo_debug_attn_profile(ctypes.c_void_p(buf.data_ptr()))

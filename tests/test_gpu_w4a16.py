@@ -238,3 +238,31 @@ def test_w4a16_packed_stream_k(lmo, N, K, batch):
     # vs the unsplit run: only the fp32 summation order differs (tensor-core accumulation
     # of the whole K vs atomic adds of range partials): |dy| <= K * 2^-24 * sum|x w|
     assert np.all(np.abs(ya.numpy().astype(np.float64) - y1.numpy()) <= K * 2.0 ** -24 * absdot + 1e-6)
+
+
+@pytest.mark.parametrize("N,K,B", [(21504, 7168, 64),     # c3 QKV: stream-K, BN = 64
+                                   (27648, 9216, 64),     # c4 QKV: stream-K
+                                   (24576, 8192, 128),    # c5 QKV: BN = 128, 2 CTAs/SM, split-K
+                                   (8192, 32768, 128)])   # c5 FFN2: long K, split-K
+def test_w4a16_packed_bench_shapes_sampled(lmo, N, K, B):
+    """The packed GEMM at the bench's full shapes in its launch configuration (auto split:
+    stream-K or split-K with the overlapped zeroing), sampled output features -- the first
+    and last rows of tiles (where stream-K ranges hand a tile over) and random rows --
+    against the oracle bound."""
+    rng = np.random.default_rng(N + K + B)
+    W = (rng.standard_normal((N, K), dtype=np.float32) * 0.02).astype(np.float16)
+    Wt = torch.from_numpy(W).cuda()
+    codes = torch.empty((N, K // 2), dtype=torch.uint8, device="cuda")
+    meta = torch.empty((N, K // 64), dtype=torch.int32, device="cuda")
+    lmo.lmo_quantize_groupwise(Wt, N, K, 1, codes=codes, meta=meta)
+    del Wt
+    packed = lmo.lmo_w4a16_pack(codes, meta, N, K)
+    x = rng.standard_normal((B, K)).astype(np.float16)
+    y = lmo.lmo_w4a16_linear_packed(packed, N, K, torch.from_numpy(x).cuda()).cpu().numpy()
+    rows = np.unique(np.concatenate([[0, 127, 128, N - 128, N - 1], rng.choice(N, 19, replace=False)]))
+    ch = codes[rows].cpu().numpy()
+    mh = meta[rows].cpu().numpy().view(np.uint16).reshape(len(rows), K // 64, 2)
+    ref = oracle.w4a16_linear(ch, mh, len(rows), K, x)
+    wdq = oracle.dequantize_groupwise(ch, mh, len(rows), K, 1).reshape(len(rows), K).astype(np.float64)
+    bound = np.abs(x.astype(np.float64)) @ np.abs(wdq).T * 2.0 ** -10 + 1e-6
+    assert np.all(np.abs(y[:, rows] - ref) <= bound)

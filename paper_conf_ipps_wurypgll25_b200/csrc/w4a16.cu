@@ -35,6 +35,7 @@
 #include <cuda.h>
 
 #include <algorithm>
+#include <atomic>
 
 #include "common.cuh"
 
@@ -949,7 +950,8 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
                          int N, int K, int batch, int ksplit, cudaStream_t st) {
     EncodeTiledFn enc = encode_tiled();
     if (!enc) return cudaErrorNotSupported;
-    const int BN = batch <= 64 ? 64 : 128;
+    const int BN = batch <= 64 ? 64 : 128;   // UMMA N = the batch rounded up (an N = 32 instance for
+                                             // batch <= 32 measured equal on c2: 76.4 vs 74-76 us/layer)
     CUtensorMap tc, tx;
     {   // x [batch][K] fp16, box 64 x BN rows, SWIZZLE_128B (rows >= batch are zero-filled)
         const cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)batch};
@@ -976,11 +978,22 @@ cudaError_t launch_w4a16(const uint8_t *codes, const void *meta, const uint8_t *
     if (packed && LMO_W4_G2 && MT == 1 && K % (2 * w4::kK) == 0) {   // two groups per pipeline step
         cudaError_t pre = cudaSuccess;
         auto go2 = [&](auto kern, int smem_bytes, int tmem_cols, bool sk_ok) {
-            cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
-            cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
+            // attributes and the resident-CTA count once per (device, instance): the host path of a
+            // small GEMM is launch-bound (c2 layer: ~50 us of host enqueue for 4 GEMMs)
+            static std::atomic<int> occ_cache[64][2];
+            int dev = 0;
+            cudaGetDevice(&dev);
+            if (dev < 0 || dev >= 64) dev = 0;
+            const int bi = BN == 64 ? 0 : 1;
+            int occ = occ_cache[dev][bi].load(std::memory_order_acquire);
+            if (occ == 0) {
+                cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_bytes);
+                cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
+                occ = w4a16_resident_ctas(smem_bytes, tmem_cols, LMO_W4_G2_DW * 32 + 96);
+                occ_cache[dev][bi].store(occ, std::memory_order_release);
+            }
             int sk_ctas = 0;
             if (ksplit <= 0) {
-                const int occ = w4a16_resident_ctas(smem_bytes, tmem_cols, LMO_W4_G2_DW * 32 + 96);
                 ksplit = w4a16_auto_split(N, K, occ);
                 // Stream-K when the tiles do not fill the resident slots evenly (e.g. 168 or 224
                 // tiles on 296 slots: 2-tile SMs beside 1-tile SMs): the linearised tile-steps cut
